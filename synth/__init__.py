@@ -1,0 +1,178 @@
+"""Seeded synthetic SDRBench-shaped fields (inputs only -- no codec arithmetic).
+
+Shared by tests/ and bench.py; imported by neither the oracle nor the CUDA
+path.  The paper's inputs (Table II) are smooth, centred around
+zero and free of denormals/NaN/inf; the datasets themselves are not
+available (no network), so DESIGN.md section 6 defines this recipe:
+
+    g(x) = sum_{m=1..32} a_m sin(2 pi k_m . x^ + phi_m)        (unit RMS)
+    field = A * g(x) + A * tau * h(idx)
+
+with integer wave vectors k_m in [-6,6]^d \\ {0}, a_m ~ |k_m|^-2, phases
+U[0, 2pi), all drawn from numpy.random.default_rng(seed); x^ = grid
+coordinates normalised to [0,1); h = a 32-bit integer hash of the linear
+index mapped to U[-1,1) (deterministic "texture").  Evaluated in float64
+with torch on any device, then cast; generation is slab-wise along the
+slowest axis so 2^32-element fields never need a float64 copy.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field as dc_field
+
+import numpy as np
+import torch
+
+
+@dataclass(frozen=True)
+class FieldSpec:
+    name: str
+    shape: tuple
+    dtype: str            # "f32" | "f64"
+    seed: int
+    A: float = 1.0        # amplitude
+    tau: float = 0.0      # texture amplitude relative to A
+    offset: float = 0.0   # additive constant (before zero masking)
+    zero_frac: float = 0.0  # fraction of the slowest axis set to exact 0.0 (REL zero path)
+    notes: str = ""
+
+    @property
+    def n(self) -> int:
+        return int(np.prod(self.shape))
+
+    @property
+    def itemsize(self) -> int:
+        return 4 if self.dtype == "f32" else 8
+
+    @property
+    def nbytes(self) -> int:
+        return self.n * self.itemsize
+
+
+# Calibrated so the f32 ABS 1E-3 ratio of the CESM/NYX shapes lands near the
+# paper's geo-mean range (14 at 1E-4 ... 68 at 1E-1); see DESIGN.md 6.
+CONFIGS = {
+    "cesm": FieldSpec("CESM-ATM-shaped 1800x3600 f32", (1800, 3600), "f32", 1, A=0.3, tau=1e-3),
+    "nyx": FieldSpec("NYX-shaped 512^3 f32", (512, 512, 512), "f32", 2, A=0.02, tau=1e-3),
+    # "rough" variant (ratio ~4-5 at ABS 1E-3): more active bit planes per chunk
+    "nyx_rough": FieldSpec("NYX-shaped 512^3 f32 (rough)", (512, 512, 512), "f32", 2,
+                           A=2.0, tau=1e-3),
+    "hurricane": FieldSpec("Hurricane-shaped 100x500x500 f32", (100, 500, 500), "f32", 3,
+                           A=10.0, tau=1e-4, zero_frac=0.05),
+    "miranda": FieldSpec("Miranda-shaped 256x384x384 f64", (256, 384, 384), "f64", 6,
+                         A=1.0, tau=1e-6, offset=2.0),
+    "big16g": FieldSpec("16 GiB f32 field 1024x2048x2048", (1024, 2048, 2048), "f32", 7,
+                        A=0.02, tau=1e-3),
+}
+
+
+def _modes(ndim: int, seed: int, nmodes: int = 32):
+    rng = np.random.default_rng(seed)
+    ks = []
+    while len(ks) < nmodes:
+        k = rng.integers(-6, 7, size=ndim)
+        if np.any(k != 0):
+            ks.append(k)
+    ks = np.array(ks, dtype=np.float64)
+    amp = 1.0 / np.sum(ks * ks, axis=1)
+    amp = amp / math.sqrt(np.sum(amp * amp) / 2.0)      # unit RMS
+    phi = rng.uniform(0.0, 2.0 * math.pi, size=nmodes)
+    return ks, amp, phi
+
+
+def _hash_u01(idx: torch.Tensor) -> torch.Tensor:
+    """32-bit integer hash of int64 indices -> float64 in [-1, 1)."""
+    M = 0xFFFFFFFF
+    x = (idx ^ (idx >> 32)) & M
+    x = x ^ (x >> 16)
+    x = (x * 0x7FEB352D) & M
+    x = x ^ (x >> 15)
+    x = (x * 0x846CA68B) & M
+    x = x ^ (x >> 16)
+    return x.to(torch.float64) * (2.0 / 4294967296.0) - 1.0
+
+
+def generate(spec: FieldSpec, device="cpu", slab: tuple | None = None,
+             max_slab_elems: int = 1 << 25) -> torch.Tensor:
+    """Return the field (or rows [slab[0], slab[1]) of its slowest axis) flat.
+
+    The result is a contiguous 1-D tensor of dtype float32/float64 on `device`.
+    """
+    shape = spec.shape
+    nd = len(shape)
+    ks, amp, phi = _modes(nd, spec.seed)
+    lo, hi = (0, shape[0]) if slab is None else slab
+    inner = int(np.prod(shape[1:])) if nd > 1 else 1
+    tdt = torch.float32 if spec.dtype == "f32" else torch.float64
+    out = torch.empty((hi - lo) * inner, dtype=tdt, device=device)
+    rows_per = max(1, max_slab_elems // inner)
+    kt = torch.tensor(ks, dtype=torch.float64, device=device)
+    at = torch.tensor(amp, dtype=torch.float64, device=device)
+    pt = torch.tensor(phi, dtype=torch.float64, device=device)
+    zero_rows = int(round(spec.zero_frac * shape[0]))
+    for r0 in range(lo, hi, rows_per):
+        r1 = min(hi, r0 + rows_per)
+        axes = [torch.arange(r0, r1, dtype=torch.float64, device=device) / shape[0]]
+        for d in range(1, nd):
+            axes.append(torch.arange(shape[d], dtype=torch.float64, device=device) / shape[d])
+        grids = torch.meshgrid(*axes, indexing="ij")
+        g = torch.zeros(grids[0].shape, dtype=torch.float64, device=device)
+        for m in range(ks.shape[0]):
+            arg = pt[m].clone()
+            arg = arg + 2.0 * math.pi * sum(kt[m, d] * grids[d] for d in range(nd))
+            g += at[m] * torch.sin(arg)
+        vals = spec.A * g.reshape(-1) + spec.offset
+        if spec.tau:
+            idx = torch.arange(r0 * inner, r1 * inner, dtype=torch.int64, device=device)
+            vals = vals + spec.A * spec.tau * _hash_u01(idx)
+        if zero_rows:
+            # exact zeros in a block of the slowest axis (REL lossless-zero path)
+            zr0, zr1 = shape[0] // 2, shape[0] // 2 + zero_rows
+            a, b = max(r0, zr0), min(r1, zr1)
+            if a < b:
+                vals[(a - r0) * inner:(b - r0) * inner] = 0.0
+        out[(r0 - lo) * inner:(r1 - lo) * inner] = vals.to(tdt)
+    return out
+
+
+def chunk_slab(spec: FieldSpec, rank: int, world: int, chunk_bytes: int = 16384):
+    """Chunk-aligned element range [e0, e1) owned by `rank`."""
+    cw = chunk_bytes // spec.itemsize
+    C = (spec.n + cw - 1) // cw
+    c0, c1 = rank * C // world, (rank + 1) * C // world
+    return c0 * cw, min(c1 * cw, spec.n)
+
+
+def adversarial_f32(n: int = 4099, seed: int = 8) -> np.ndarray:
+    """Special values for correctness tests: +-0, denormals, FLT_MIN/MAX, inf,
+    NaNs with payloads and both signs, huge alternating ranges (the cuSZp
+    pre-quantisation overflow case), and ordinary values."""
+    rng = np.random.default_rng(seed)
+    specials = np.array([0x00000000, 0x80000000, 0x00000001, 0x80000001, 0x007FFFFF,
+                         0x807FFFFF, 0x00800000, 0x80800000, 0x7F7FFFFF, 0xFF7FFFFF,
+                         0x7F800000, 0xFF800000, 0x7FC00000, 0xFFC00000, 0x7F800001,
+                         0xFF800001, 0x7FFFFFFF, 0xFFFFFFFF, 0x7FA12345, 0xFFB54321,
+                         0x3F800000, 0xBF800000, 0x7E800000, 0x01000000],
+                        dtype=np.uint32).view(np.float32)
+    body = rng.standard_normal(n).astype(np.float32)
+    body[::7] = specials[rng.integers(0, len(specials), size=len(body[::7]))]
+    body[1::11] = np.where(rng.random(len(body[1::11])) < 0.5, 1e38, -1e-38).astype(np.float32)
+    with np.errstate(over="ignore", invalid="ignore"):
+        body[2::13] *= np.float32(1e30)
+    body[:len(specials)] = specials
+    return body
+
+
+def adversarial_f64(n: int = 2051, seed: int = 9) -> np.ndarray:
+    rng = np.random.default_rng(seed)
+    specials = np.array([0x0000000000000000, 0x8000000000000000, 0x0000000000000001,
+                         0x800FFFFFFFFFFFFF, 0x0010000000000000, 0x7FEFFFFFFFFFFFFF,
+                         0xFFEFFFFFFFFFFFFF, 0x7FF0000000000000, 0xFFF0000000000000,
+                         0x7FF8000000000000, 0xFFF8000000000000, 0x7FF0000000000001,
+                         0xFFF0000000000001, 0xFFFFFFFFFFFFFFFF, 0x3FF0000000000000,
+                         0xBFF0000000000000], dtype=np.uint64).view(np.float64)
+    body = rng.standard_normal(n)
+    body[::7] = specials[rng.integers(0, len(specials), size=len(body[::7]))]
+    body[1::11] = np.where(rng.random(len(body[1::11])) < 0.5, 1e300, -1e-300)
+    body[:len(specials)] = specials
+    return body
