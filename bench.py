@@ -1,0 +1,413 @@
+#!/usr/bin/env python3
+"""PFPL hot-path benchmark (BASELINE.json metric).
+
+python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                [--config nyx] [--bound abs] [--eps 1e-3]
+
+One step = one pass of the whole hot path over the synthetic field: compress
+(a0-a8: quantize/verify, delta+negabinary, bit shuffle, zero/repeat
+elimination, look-back concatenation) then decompress (d1-d5).  Inputs are
+resident in HBM before timing; they are larger than L2 (NYX: 537 MB vs 126 MB)
+so no flush is needed.  Times are CUDA events on the launching stream,
+max over ranks.  value = compression throughput in uncompressed GB/s (10^9,
+P:225), whole job; decompression GB/s and ratio are reported beside it.
+
+N > 1 (torchrun, one process per GPU): weak scaling -- rank r compresses
+chunk-aligned slab r of an (N*512)x512x512 field; NCCL all-reduces the NOA
+range (NOA only) and all-gathers the per-shard payload sizes so every rank
+knows its offset in the single assembled stream.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "compress/decompress GB/s (uncompressed) + ratio, f32 ABS 1E-3, 1/2/4/8 B200"
+PAPER_CONTEXT = {"paper_pfpl_cuda_rtx4090_gbs": 423, "paper_pfpl_omp_ryzen2950x_gbs": 5,
+                 "note": "f32 ABS 1E-3 SDRBench geo-mean (P:15); other hardware, context only"}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="nyx")
+    ap.add_argument("--bound", default="abs")
+    ap.add_argument("--eps", type=float, default=1e-3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--quiet", action="store_true")
+    return ap.parse_args()
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return None
+
+
+class Clocks:
+    """Sample nvidia-smi clocks/throttle reasons during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def cpu_baseline(spec, bound, eps, seconds):
+    """The oracle as it stands (plain C, chunks over all host threads) on a
+    bounded sample of the same workload: the first rows of the field."""
+    import numpy as np
+    import oracle
+    import synth
+    cores = len(os.sched_getaffinity(0))
+    oracle.build()
+    inner = spec.n // spec.shape[0]
+    rows = max(1, min(spec.shape[0], (64 << 20) // (inner * spec.itemsize)))
+    x = synth.generate(spec, slab=(0, rows)).numpy()
+    t0 = time.perf_counter()
+    s = oracle.compress(x, bound, eps, nthreads=cores)
+    t1 = time.perf_counter()
+    reps = max(1, int(seconds / max(t1 - t0, 1e-3)))
+    reps = min(reps, 50)
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        oracle.compress(x, bound, eps, nthreads=cores)
+    tc = (time.perf_counter() - t0) / reps
+    t0 = time.perf_counter()
+    for _ in range(max(1, reps // 2)):
+        oracle.decompress(s, nthreads=cores)
+    td = (time.perf_counter() - t0) / max(1, reps // 2)
+    return {"value": x.nbytes / tc / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {rows} of {spec.shape[0]} rows ({x.nbytes / 1e6:.1f} MB), "
+                      f"{reps} reps, OpenMP over chunks",
+            "decompress_gbs": x.nbytes / td / 1e9, "ratio": x.nbytes / len(s)}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle, timed on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    import synth
+    spec = synth.CONFIGS[args.config]
+    cores = len(os.sched_getaffinity(0))
+    oracle.build()
+    inner = spec.n // spec.shape[0]
+    rows = max(1, min(spec.shape[0], (32 << 20) // (inner * spec.itemsize)))
+    x = synth.generate(spec, slab=(0, rows)).numpy()
+    for _ in range(args.warmup):
+        s = oracle.compress(x, args.bound, args.eps, nthreads=cores)
+    tc, td = [], []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        s = oracle.compress(x, args.bound, args.eps, nthreads=cores)
+        t1 = time.perf_counter()
+        oracle.decompress(s, nthreads=cores)
+        t2 = time.perf_counter()
+        tc.append(t1 - t0)
+        td.append(t2 - t1)
+    comp = x.nbytes / statistics.median(tc) / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": comp, "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * (statistics.median(tc) + statistics.median(td)),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": spec.dtype,
+        "data": "synthetic", "config": _config(spec, args, sample_rows=rows),
+        "ratio": x.nbytes / len(s), "decompress_gbs": x.nbytes / statistics.median(td) / 1e9,
+        "cpu_baseline": {"value": comp, "unit": "GB/s", "cores": cores, "kind": "oracle",
+                         "sample": f"first {rows} of {spec.shape[0]} rows ({x.nbytes / 1e6:.1f} MB) per step"},
+        "e2e": {"value": comp, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "context": PAPER_CONTEXT,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def _config(spec, args, sample_rows=None):
+    c = {"workload": f"{spec.name}, {args.bound.upper()} {args.eps:g}", "shape": list(spec.shape),
+         "bound": args.bound, "eps": args.eps, "n": spec.n, "bytes": spec.nbytes,
+         "l2": "inputs larger than L2 (no flush needed)" if spec.nbytes > 126e6 else "L2 flushed",
+         "parallelism": f"dp{args.gpus} chunk shards"}
+    if sample_rows is not None:
+        c["sample_rows"] = sample_rows
+    return c
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_fallinadcb25_b200 as pk
+    import synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_ipps_fallinadcb25_b200 import _build
+    if rank == 0:
+        _build.build()
+    if world > 1:
+        dist.barrier()
+    L = pk.lib()
+
+    base = synth.CONFIGS[args.config]
+    if world > 1:
+        import dataclasses
+        spec = dataclasses.replace(base, shape=(base.shape[0] * world,) + tuple(base.shape[1:]))
+        x = synth.generate(spec, device=dev, slab=(rank * base.shape[0], (rank + 1) * base.shape[0]))
+    else:
+        spec = base
+        x = synth.generate(spec, device=dev)
+    torch.cuda.synchronize()
+    n = x.numel()
+    esz = x.element_size()
+    nbytes = n * esz
+    cw = 16384 // esz
+    C = -(-n // cw)
+    dt = pk.F32 if x.dtype == torch.float32 else pk.F64
+    bd = pk._BOUNDS[args.bound]
+    stream = torch.cuda.current_stream()
+    sh = stream.cuda_stream
+    cap = pk.max_compressed_bytes(n, dt)
+    out = torch.empty(cap, dtype=torch.uint8, device=dev)
+    res = torch.zeros(4, dtype=torch.int64, device=dev)
+    y = torch.empty_like(x)
+    first_chunk = rank * C
+    n_total = n * world
+    mm = torch.empty(2, dtype=torch.float64, device=dev)
+    sizes = torch.zeros(world, dtype=torch.int64, device=dev)
+    import ctypes
+
+    # ---- one step = compress then decompress ----
+    def compress_once():
+        if world == 1:
+            pk._check(L.pfpl_compress_async(x.data_ptr(), n, dt, bd, args.eps, 0, out.data_ptr(), cap,
+                                            res.data_ptr(), sh))
+        else:
+            if bd == pk.NOA:
+                pk._check(L.pfpl_minmax(x.data_ptr(), n, dt, mm.data_ptr(), sh))
+                v = torch.stack([mm[1], -mm[0]])
+                dist.all_reduce(v, op=dist.ReduceOp.MAX)
+                mm[0] = -v[1]
+                mm[1] = v[0]
+            pb = ctypes.c_uint64(0)
+            pk._check(L.pfpl_compress_shard(x.data_ptr(), n, first_chunk, n_total, dt, bd, args.eps,
+                                            0, mm.data_ptr() if bd == pk.NOA else None,
+                                            out.data_ptr(), cap, ctypes.byref(pb), None, sh))
+            sizes[rank] = pb.value
+            dist.all_gather_into_tensor(sizes, sizes[rank:rank + 1].clone())
+            return int(pb.value)
+        return None
+
+    hdr = None
+
+    def decompress_once(pbytes):
+        nonlocal hdr
+        if world == 1:
+            pk._check(L.pfpl_decompress_async(out.data_ptr(), int(res_bytes), hdr_buf, y.data_ptr(),
+                                              nbytes, res.data_ptr(), sh))
+        else:
+            pk._check(L.pfpl_decompress_chunks(hdr_buf, table_host.ctypes.data_as(ctypes.c_void_p),
+                                               first_chunk, C, out.data_ptr() + 4 * C, pbytes,
+                                               y.data_ptr(), nbytes, sh))
+
+    # warm-up (also fixes the header / table for the decompress leg)
+    for _ in range(max(1, args.warmup)):
+        pb = compress_once()
+    torch.cuda.synchronize()
+    if world == 1:
+        res_bytes = int(res[0].item())
+        hdr_bytes = out[:48].cpu().numpy().tobytes()
+        comp_bytes = res_bytes
+    else:
+        import numpy as np
+        table_host = out[:4 * C].cpu().numpy().view(np.uint32).copy()
+        hdr_bytes = None
+        # header from the shard call (identical on every rank)
+        hb = ctypes.create_string_buffer(48)
+        pb2 = ctypes.c_uint64(0)
+        pk._check(L.pfpl_compress_shard(x.data_ptr(), n, first_chunk, n_total, dt, bd, args.eps, 0,
+                                        mm.data_ptr() if bd == pk.NOA else None, out.data_ptr(), cap,
+                                        ctypes.byref(pb2), ctypes.cast(hb, ctypes.c_void_p), sh))
+        hdr_bytes = hb.raw
+        comp_bytes = 48 / world + 4 * C + pb2.value
+    hdr_buf = ctypes.cast(ctypes.create_string_buffer(hdr_bytes, 48), ctypes.c_void_p)
+    for _ in range(max(1, args.warmup)):
+        decompress_once(pb if world > 1 else None)
+    torch.cuda.synchronize()
+    if world == 1:
+        assert int(res[1].item()) == 0, "decode reported corruption"
+
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    launches0 = pk.launch_count()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with Clocks(local) as clk:
+        t_wall0 = time.perf_counter()
+        for i in range(args.steps):
+            ev[i][0].record(stream)
+            pb = compress_once()
+            ev[i][1].record(stream)
+            decompress_once(pb)
+            ev[i][2].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t_wall = time.perf_counter() - t_wall0
+    launches = pk.launch_count() - launches0
+    tc = [ev[i][0].elapsed_time(ev[i][1]) for i in range(args.steps)]
+    td = [ev[i][1].elapsed_time(ev[i][2]) for i in range(args.steps)]
+    tc_sum, td_sum = sum(tc), sum(td)
+    if world > 1:
+        t = torch.tensor([tc_sum, td_sum], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tc_sum, td_sum = t.tolist()
+        comp_total = torch.tensor([comp_bytes], dtype=torch.float64, device=dev)
+        dist.all_reduce(comp_total)
+        comp_bytes_all = comp_total.item()
+    else:
+        comp_bytes_all = comp_bytes
+    total_bytes = nbytes * world
+    comp_gbs = total_bytes * args.steps / (tc_sum * 1e-3) / 1e9
+    dec_gbs = total_bytes * args.steps / (td_sum * 1e-3) / 1e9
+    ratio = total_bytes / comp_bytes_all
+
+    # ---- roofline of the dominant kernel (the fused encoder), measured live ----
+    peaks = _peaks()
+    peak = peaks["hbm_gbs"] if peaks else 6650.0
+    enc_ms = statistics.median(tc)
+    algo = nbytes + comp_bytes              # input read + stream written, per launch
+    roof = {"bound": "hbm", "achieved": algo / (enc_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+            "frac": algo / (enc_ms * 1e-3) / 1e9 / peak, "traffic": None,
+            "kernel": "encode_kernel (compress step)",
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s (B200_PROFILING.md)"}
+    dec_ms = statistics.median(td)
+    roof_dec = {"achieved": algo / (dec_ms * 1e-3) / 1e9, "frac": algo / (dec_ms * 1e-3) / 1e9 / peak}
+
+    # ---- end to end through the C ABI with host buffers (pinned) ----
+    e2e = None
+    if world == 1:
+        xh = x.cpu().pin_memory()
+        oh = torch.empty(cap, dtype=torch.uint8).pin_memory()
+        xd2 = torch.empty_like(x)
+        e_steps = max(2, min(args.steps, 5))
+        t0e = torch.cuda.Event(enable_timing=True)
+        t1e = torch.cuda.Event(enable_timing=True)
+        d2h = 0
+        for it in range(e_steps + 1):
+            if it == 1:
+                t0e.record(stream)
+            xd2.copy_(xh, non_blocking=True)
+            nb = ctypes.c_uint64(cap)
+            pk._check(L.pfpl_compress(xd2.data_ptr(), n, dt, bd, args.eps, out.data_ptr(),
+                                      ctypes.byref(nb), sh))
+            oh[:nb.value].copy_(out[:nb.value], non_blocking=True)
+            d2h = nb.value
+        t1e.record(stream)
+        torch.cuda.synchronize()
+        e_ms = t0e.elapsed_time(t1e) / e_steps
+        e2e = {"value": nbytes / (e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
+               "d2h_bytes_per_step": int(d2h), "what": "pinned H2D of the field + pfpl_compress + D2H of the stream"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+    line = {
+        "metric": METRIC, "value": comp_gbs, "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": (tc_sum + td_sum) / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": spec.dtype, "data": "synthetic",
+        "config": _config(base, args),
+        "ratio": ratio, "compress_gbs": comp_gbs, "decompress_gbs": dec_gbs,
+        "compress_ms": tc_sum / args.steps, "decompress_ms": td_sum / args.steps,
+        "roofline": roof, "roofline_decode": roof_dec,
+        "gpu_launches": int(launches), "launches_per_step": launches / args.steps,
+        "clocks": clk.summary(), "wall_s": t_wall, "e2e": e2e, "context": PAPER_CONTEXT,
+    }
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(base, args.bound, args.eps, args.cpu_seconds)
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,230 @@
+"""PFPL hot path on B200 -- thin Python binding of libpfpl.so (include/pfpl.h).
+
+Argument marshalling only: every step of compression and decompression runs
+in the sm_100a kernels behind the C ABI.  torch supplies device memory and
+streams.  There is no CPU fallback: if the CUDA library or a GPU is missing,
+every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+from . import _build
+
+__all__ = ["compress", "decompress", "compress_async", "decompress_async", "minmax",
+           "compress_shard", "decompress_chunks", "peek_header", "max_compressed_bytes",
+           "PFPLError", "lib", "launch_count"]
+
+F32, F64 = 0, 1
+ABS, REL, NOA = 0, 1, 2
+OPT_MS = 2
+HEADER_BYTES = 48
+CHUNK_BYTES = 16384
+_BOUNDS = {"abs": ABS, "rel": REL, "noa": NOA}
+_ERR = {-1: "invalid argument", -2: "invalid error bound", -3: "output capacity too small",
+        -4: "corrupt stream", -5: "buffer not 16-byte aligned", -6: "CUDA runtime error"}
+
+
+class PFPLError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        super().__init__(f"pfpl error {code} ({_ERR.get(code, '?')}) {what}".strip())
+        self.code = code
+
+
+_lib = None
+
+
+def lib():
+    """Load libpfpl.so (built in-tree by __graft_entry__.build())."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_build.LIB):
+            raise PFPLError(-6, f"{_build.LIB} is missing; run __graft_entry__.build()")
+        L = ctypes.CDLL(_build.LIB)
+        vp, u64, i32, dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
+        pu64 = ctypes.POINTER(ctypes.c_uint64)
+        sig = {
+            "pfpl_max_compressed_bytes": (u64, [u64, i32]),
+            "pfpl_compress": (i32, [vp, u64, i32, i32, dbl, vp, pu64, vp]),
+            "pfpl_compress_ex": (i32, [vp, u64, i32, i32, dbl, ctypes.c_uint, vp, pu64, vp]),
+            "pfpl_compress_async": (i32, [vp, u64, i32, i32, dbl, ctypes.c_uint, vp, u64, vp, vp]),
+            "pfpl_decompress": (i32, [vp, u64, vp, pu64, vp]),
+            "pfpl_decompress_async": (i32, [vp, u64, vp, vp, u64, vp, vp]),
+            "pfpl_peek_header": (i32, [vp, u64, pu64, ctypes.POINTER(i32), ctypes.POINTER(i32),
+                                       ctypes.POINTER(dbl), ctypes.POINTER(ctypes.c_uint)]),
+            "pfpl_minmax": (i32, [vp, u64, i32, vp, vp]),
+            "pfpl_compress_shard": (i32, [vp, u64, u64, u64, i32, i32, dbl, ctypes.c_uint, vp, vp,
+                                          u64, pu64, vp, vp]),
+            "pfpl_decompress_chunks": (i32, [vp, vp, u64, u64, vp, u64, vp, u64, vp]),
+            "pfpl_strerror": (ctypes.c_char_p, [i32]),
+            "pfpl_last_cuda_error": (i32, []),
+            "pfpl_release_scratch": (i32, []),
+            "pfpl_launch_count": (u64, []),
+            "pfpl_version": (ctypes.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype, f.argtypes = res, args
+        _lib = L
+    return _lib
+
+
+def _check(st: int, what: str = ""):
+    if st != 0:
+        extra = ""
+        if st == -6:
+            extra = f"cudaError={lib().pfpl_last_cuda_error()}"
+        raise PFPLError(st, (what + " " + extra).strip())
+
+
+def _stream(stream) -> int:
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    if t.dtype == torch.float32:
+        return F32
+    if t.dtype == torch.float64:
+        return F64
+    raise TypeError(f"PFPL compresses float32/float64, got {t.dtype}")
+
+
+def _bound(b) -> int:
+    return _BOUNDS[b.lower()] if isinstance(b, str) else int(b)
+
+
+def _require_cuda(t: torch.Tensor, name: str):
+    if not t.is_cuda:
+        raise PFPLError(-1, f"{name} must be a CUDA tensor (no CPU fallback)")
+    if not t.is_contiguous():
+        raise PFPLError(-1, f"{name} must be contiguous")
+
+
+def max_compressed_bytes(n: int, dtype) -> int:
+    code = dtype if isinstance(dtype, int) else (F32 if dtype in (torch.float32, "f32") else F64)
+    return int(lib().pfpl_max_compressed_bytes(n, code))
+
+
+def compress(x: torch.Tensor, bound="abs", eps: float = 1e-3, ms: bool = False,
+             out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Compress a float32/float64 CUDA tensor; returns a uint8 CUDA tensor (a
+    view of `out` if given) holding the stream."""
+    _require_cuda(x, "x")
+    dt = _dtype_code(x)
+    n = x.numel()
+    cap = max_compressed_bytes(n, dt)
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, device=x.device)
+    nbytes = ctypes.c_uint64(out.numel())
+    with torch.cuda.device(x.device):
+        st = lib().pfpl_compress_ex(x.data_ptr(), n, dt, _bound(bound), float(eps),
+                                    OPT_MS if ms else 0, out.data_ptr(), ctypes.byref(nbytes),
+                                    _stream(stream))
+    _check(st, "compress")
+    return out[:nbytes.value]
+
+
+def compress_async(x: torch.Tensor, out: torch.Tensor, result: torch.Tensor, bound="abs",
+                   eps: float = 1e-3, ms: bool = False, stream=None) -> None:
+    """Enqueue compression without synchronising; result (int64 CUDA tensor of
+    >= 2 elements) receives [stream bytes, status]."""
+    _require_cuda(x, "x")
+    dt = _dtype_code(x)
+    st = lib().pfpl_compress_async(x.data_ptr(), x.numel(), dt, _bound(bound), float(eps),
+                                   OPT_MS if ms else 0, out.data_ptr(), out.numel(),
+                                   result.data_ptr(), _stream(stream))
+    _check(st, "compress_async")
+
+
+def peek_header(hdr: bytes):
+    n = ctypes.c_uint64()
+    dt = ctypes.c_int()
+    bd = ctypes.c_int()
+    eps = ctypes.c_double()
+    fl = ctypes.c_uint()
+    buf = ctypes.create_string_buffer(bytes(hdr[:HEADER_BYTES]), HEADER_BYTES)
+    _check(lib().pfpl_peek_header(ctypes.cast(buf, ctypes.c_void_p), len(hdr), ctypes.byref(n),
+                                  ctypes.byref(dt), ctypes.byref(bd), ctypes.byref(eps),
+                                  ctypes.byref(fl)), "peek_header")
+    return {"n": n.value, "dtype": dt.value, "bound": bd.value, "eps": eps.value, "flags": fl.value}
+
+
+def decompress(buf: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Decompress a uint8 CUDA tensor holding a stream."""
+    _require_cuda(buf, "buf")
+    if buf.numel() < HEADER_BYTES:
+        raise PFPLError(-4, "stream shorter than its header")
+    hdr = buf[:HEADER_BYTES].cpu().numpy().tobytes()
+    h = peek_header(hdr)
+    tdt = torch.float32 if h["dtype"] == F32 else torch.float64
+    if out is None:
+        out = torch.empty(max(h["n"], 1), dtype=tdt, device=buf.device)
+    ob = ctypes.c_uint64(out.numel() * out.element_size())
+    with torch.cuda.device(buf.device):
+        st = lib().pfpl_decompress(buf.data_ptr(), buf.numel(), out.data_ptr(), ctypes.byref(ob),
+                                   _stream(stream))
+    _check(st, "decompress")
+    return out[:h["n"]]
+
+
+def decompress_async(buf: torch.Tensor, hdr: bytes, out: torch.Tensor, result: torch.Tensor,
+                     stream=None) -> None:
+    h = ctypes.create_string_buffer(bytes(hdr[:HEADER_BYTES]), HEADER_BYTES)
+    st = lib().pfpl_decompress_async(buf.data_ptr(), buf.numel(), ctypes.cast(h, ctypes.c_void_p),
+                                     out.data_ptr(), out.numel() * out.element_size(),
+                                     result.data_ptr(), _stream(stream))
+    _check(st, "decompress_async")
+
+
+def minmax(x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """{min, max} over the finite elements (NOA step) as a float64 CUDA tensor."""
+    _require_cuda(x, "x")
+    if out is None:
+        out = torch.empty(2, dtype=torch.float64, device=x.device)
+    _check(lib().pfpl_minmax(x.data_ptr(), x.numel(), _dtype_code(x), out.data_ptr(),
+                             _stream(stream)), "minmax")
+    return out
+
+
+def compress_shard(x: torch.Tensor, first_chunk: int, n_total: int, bound="abs",
+                   eps: float = 1e-3, ms: bool = False, mnmx: torch.Tensor | None = None,
+                   out: torch.Tensor | None = None, stream=None):
+    """Compress a chunk-aligned shard. Returns (table_u32 view, payload view, header bytes)."""
+    _require_cuda(x, "x")
+    dt = _dtype_code(x)
+    n = x.numel()
+    C = -(-n * x.element_size() // CHUNK_BYTES)
+    cap = 4 * C + n * x.element_size() + 16
+    if out is None:
+        out = torch.empty(cap, dtype=torch.uint8, device=x.device)
+    pb = ctypes.c_uint64(0)
+    hdr = ctypes.create_string_buffer(HEADER_BYTES)
+    st = lib().pfpl_compress_shard(x.data_ptr(), n, first_chunk, n_total, dt, _bound(bound),
+                                   float(eps), OPT_MS if ms else 0,
+                                   mnmx.data_ptr() if mnmx is not None else None,
+                                   out.data_ptr(), out.numel(), ctypes.byref(pb),
+                                   ctypes.cast(hdr, ctypes.c_void_p), _stream(stream))
+    _check(st, "compress_shard")
+    return out[:4 * C], out[4 * C:4 * C + pb.value], hdr.raw
+
+
+def decompress_chunks(hdr: bytes, table, first_chunk: int, payload: torch.Tensor,
+                      out: torch.Tensor, stream=None) -> None:
+    import numpy as np
+    tab = np.ascontiguousarray(np.asarray(table, dtype=np.uint32))
+    h = ctypes.create_string_buffer(bytes(hdr[:HEADER_BYTES]), HEADER_BYTES)
+    st = lib().pfpl_decompress_chunks(ctypes.cast(h, ctypes.c_void_p),
+                                      tab.ctypes.data_as(ctypes.c_void_p), first_chunk, tab.size,
+                                      payload.data_ptr() if payload.numel() else None,
+                                      payload.numel(), out.data_ptr(),
+                                      out.numel() * out.element_size(), _stream(stream))
+    _check(st, "decompress_chunks")
+
+
+def launch_count() -> int:
+    return int(lib().pfpl_launch_count())

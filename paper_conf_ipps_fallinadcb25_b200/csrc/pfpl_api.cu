@@ -1,0 +1,567 @@
+// pfpl_api.cu -- host side of the C ABI declared in include/pfpl.h.
+//
+// Validation, quantizer constants (readings R1, R4, R5 of DESIGN.md 3),
+// per-(device, stream) scratch (look-back descriptors, monotone tickets,
+// epochs), and kernel launches.  No computation of the codec happens here:
+// every step of the path runs in the kernels of pfpl_encode.cu /
+// pfpl_decode.cu / pfpl_misc.cu.
+#include <atomic>
+#include <cfloat>
+#include <cmath>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <utility>
+
+#include "../../include/pfpl.h"
+#include "pfpl_internal.h"
+
+using namespace pfpl;
+
+namespace {
+
+std::atomic<int> g_last_cuda{0};
+std::atomic<uint64_t> g_launches{0};
+
+struct Scratch {
+    unsigned long long* status = nullptr;
+    uint64_t status_cap = 0;
+    unsigned long long* ticket = nullptr;
+    uint64_t ticket_val = 0;
+    uint32_t epoch = 0;
+    QConst* qc_dev = nullptr;
+    double* mnmx = nullptr;
+    double* partial = nullptr;
+    uint64_t* result = nullptr;      // [0] stream bytes, [1] error word
+    uint64_t* host = nullptr;        // pinned mirror of result
+    uint8_t* hdr_host = nullptr;     // pinned 64 bytes
+    uint32_t* table_dev = nullptr;   // for pfpl_decompress_chunks
+    uint64_t table_cap = 0;
+};
+
+std::mutex g_mu;
+std::map<std::pair<int, void*>, Scratch*> g_scratch;
+
+constexpr int kMinmaxBlocks = 592;
+
+int cuda_fail(cudaError_t e) {
+    g_last_cuda = (int)e;
+    return PFPL_ERR_CUDA;
+}
+#define CK(x)                                             \
+    do {                                                  \
+        cudaError_t _e = (x);                             \
+        if (_e != cudaSuccess) return cuda_fail(_e);      \
+    } while (0)
+
+int get_scratch(cudaStream_t s, uint64_t C, Scratch** out) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    Scratch*& sc = g_scratch[{dev, (void*)s}];
+    if (!sc) {
+        sc = new Scratch();
+        CK(cudaMalloc(&sc->ticket, 64));
+        CK(cudaMemsetAsync(sc->ticket, 0, 64, s));
+        CK(cudaMalloc(&sc->qc_dev, sizeof(QConst)));
+        CK(cudaMalloc(&sc->mnmx, 4 * sizeof(double)));
+        CK(cudaMalloc(&sc->partial, 2 * kMinmaxBlocks * sizeof(double)));
+        CK(cudaMalloc(&sc->result, 4 * sizeof(uint64_t)));
+        CK(cudaMallocHost(&sc->host, 4 * sizeof(uint64_t)));
+        CK(cudaMallocHost(&sc->hdr_host, 64));
+    }
+    if (C > sc->status_cap) {
+        if (sc->status) CK(cudaFreeAsync(sc->status, s));
+        uint64_t cap = C < 1024 ? 1024 : C + C / 4;
+        CK(cudaMallocAsync(&sc->status, cap * sizeof(unsigned long long), s));
+        CK(cudaMemsetAsync(sc->status, 0, cap * sizeof(unsigned long long), s));
+        sc->status_cap = cap;
+        sc->epoch = 0;
+    }
+    // epochs tag look-back descriptors so no per-call memset is needed
+    if (++sc->epoch >= 0xFFFFu) {
+        CK(cudaMemsetAsync(sc->status, 0, sc->status_cap * sizeof(unsigned long long), s));
+        sc->epoch = 1;
+    }
+    *out = sc;
+    return PFPL_OK;
+}
+
+uint32_t f2u_h(float x) { uint32_t u; memcpy(&u, &x, 4); return u; }
+float u2f_h(uint32_t u) { float x; memcpy(&x, &u, 4); return x; }
+uint64_t d2u_h(double x) { uint64_t u; memcpy(&u, &x, 8); return u; }
+double u2d_h(uint64_t u) { double x; memcpy(&x, &u, 8); return x; }
+
+// R1: largest binary32 <= x (x > 0)
+float round_down_f32_h(double x) {
+    float f = (float)x;
+    if (std::isinf(f)) f = FLT_MAX;
+    if ((double)f > x) f = u2f_h(f2u_h(f) - 1u);
+    return f;
+}
+
+// quantizer constants for ABS / REL on the host (NOA is derived on the device)
+int host_qconst(int dtype, int bound, double eps, unsigned opts, QConst* qc, int* mode) {
+    memset(qc, 0, sizeof(*qc));
+    qc->flags = (opts & PFPL_OPT_MS_RESIDUALS) ? HF_MS : 0u;
+    if (!(eps > 0.0) || std::isinf(eps)) return PFPL_ERR_BOUND;
+    if (bound == PFPL_NOA) { *mode = MODE_NOA; return PFPL_OK; }
+    if (bound == PFPL_ABS) {
+        *mode = MODE_ABS;
+        if (dtype == PFPL_F32) {
+            float ee = round_down_f32_h(eps);
+            if (ee > FLT_MAX / 2) ee = FLT_MAX / 2;
+            if (!(ee >= FLT_MIN)) return PFPL_ERR_BOUND;
+            qc->a = f2u_h(ee); qc->b = f2u_h(0.5f / ee); qc->c = f2u_h(2.0f * ee); qc->qconst = f2u_h(ee);
+        } else {
+            double ee = eps;
+            if (ee > DBL_MAX / 2) ee = DBL_MAX / 2;
+            if (!(ee >= DBL_MIN)) return PFPL_ERR_BOUND;
+            qc->a = d2u_h(ee); qc->b = d2u_h(0.5 / ee); qc->c = d2u_h(2.0 * ee); qc->qconst = d2u_h(ee);
+        }
+        return PFPL_OK;
+    }
+    // REL (P:90 with R5): c_lo = largest T <= 1+eps; w = 2 log2p(c_lo); inv_w = 0.5/log2p(c_lo)
+    *mode = MODE_REL;
+    if (dtype == PFPL_F32) {
+        float c;
+        if (eps < 4503599627370496.0) {
+            c = (float)(1.0 + eps);
+            if (std::isinf(c)) c = FLT_MAX;
+            while ((double)c - 1.0 > eps) c = u2f_h(f2u_h(c) - 1u);
+        } else {
+            c = round_down_f32_h(eps);
+        }
+        const float lw = log2p_host_f32(c);
+        const float w = 2.0f * lw;
+        if (!(w > 0.0f) || std::isinf(w)) { qc->flags |= HF_RAWWORDS; *mode = MODE_RAW; return PFPL_OK; }
+        qc->a = f2u_h(c); qc->b = f2u_h(w); qc->c = f2u_h(0.5f / lw); qc->qconst = f2u_h(w);
+    } else {
+        double c;
+        if (eps < 4503599627370496.0) {
+            c = 1.0 + eps;
+            if (c - 1.0 > eps) c = u2d_h(d2u_h(c) - 1u);
+        } else {
+            c = eps;
+            if (std::isinf(c)) c = DBL_MAX;
+        }
+        const double lw = log2p_host_f64(c);
+        const double w = 2.0 * lw;
+        if (!(w > 0.0) || std::isinf(w)) { qc->flags |= HF_RAWWORDS; *mode = MODE_RAW; return PFPL_OK; }
+        qc->a = d2u_h(c); qc->b = d2u_h(w); qc->c = d2u_h(0.5 / lw); qc->qconst = d2u_h(w);
+    }
+    return PFPL_OK;
+}
+
+inline uint64_t tsz(int dtype) { return dtype == PFPL_F32 ? 4u : 8u; }
+inline uint64_t chunks_of(uint64_t n, int dtype) {
+    const uint64_t cw = kChunkBytes / tsz(dtype);
+    return (n + cw - 1) / cw;
+}
+inline bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+// Enqueue one compression (or shard) on s.  Writes stream bytes to sc->result[0].
+int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, int bound,
+                     double eps, unsigned opts, const double* mnmx_given, uint8_t* out,
+                     uint64_t cap, uint32_t* table, uint64_t payload_off, int write_header,
+                     uint64_t* result, cudaStream_t s, Scratch** sc_out) {
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return PFPL_ERR_ARG;
+    if (bound != PFPL_ABS && bound != PFPL_REL && bound != PFPL_NOA) return PFPL_ERR_ARG;
+    if (n > (1ull << 40) || n_total > (1ull << 40)) return PFPL_ERR_ARG;
+    if ((n && !in) || !out) return PFPL_ERR_ARG;
+    if (!aligned16(in) || !aligned16(out)) return PFPL_ERR_ALIGN;
+    QConst qc;
+    int mode = 0;
+    int st = host_qconst(dtype, bound, eps, opts, &qc, &mode);
+    if (st != PFPL_OK) return st;
+    const uint64_t C = chunks_of(n, dtype);
+    if (cap < payload_off) return PFPL_ERR_CAPACITY;
+    Scratch* sc = nullptr;
+    st = get_scratch(s, C, &sc);
+    if (st != PFPL_OK) return st;
+    if (sc_out) *sc_out = sc;
+    if (!result) result = sc->result;
+    const QConst* qdev = nullptr;
+    if (mode == MODE_NOA) {
+        const double* mm = mnmx_given;
+        if (!mm) {
+            CK(launch_minmax(dtype, in, n, sc->partial, kMinmaxBlocks, s));
+            CK(launch_minmax_final(sc->partial, kMinmaxBlocks, sc->mnmx, s));
+            g_launches += 2;
+            mm = sc->mnmx;
+        }
+        CK(launch_noa_derive(dtype, mm, eps, qc.flags, sc->qc_dev, s));
+        g_launches += 1;
+        qdev = sc->qc_dev;
+    }
+    if (C == 0) {
+        if (write_header) {
+            CK(launch_header_only(out, n_total, dtype, bound, eps, qc, qdev, result, s));
+        } else {
+            CK(cudaMemsetAsync(result, 0, 8, s));
+            // payload size 0 -> stream bytes = payload_off
+            uint64_t v = payload_off;
+            CK(cudaMemcpyAsync(result, &v, 8, cudaMemcpyHostToDevice, s));
+            CK(cudaStreamSynchronize(s));
+        }
+        g_launches += 1;
+        return PFPL_OK;
+    }
+    EncParams p;
+    memset(&p, 0, sizeof(p));
+    p.in = in;
+    p.n = n;
+    p.C = C;
+    p.out = out;
+    p.cap = cap;
+    p.table = table;
+    p.payload_off = payload_off;
+    p.status = sc->status;
+    p.ticket = sc->ticket;
+    p.ticket_base = sc->ticket_val;
+    p.epoch = sc->epoch;
+    p.write_header = write_header;
+    p.qc = qc;
+    p.qc_dev = qdev;
+    p.result = result;
+    p.n_total = n_total;
+    p.eps = eps;
+    p.dtype = (uint32_t)dtype;
+    p.bound = (uint32_t)bound;
+    const bool ms = (opts & PFPL_OPT_MS_RESIDUALS) != 0;
+    const int grid = encode_grid(dtype, mode, ms, C);
+    CK(launch_encode(dtype, mode, ms, p, grid, s));
+    g_launches += 1;
+    sc->ticket_val += C + (uint64_t)grid;
+    return PFPL_OK;
+}
+
+int parse_header(const uint8_t* h, uint64_t bytes, uint64_t* n, int* dtype, int* bound,
+                 double* eps, unsigned* flags, uint64_t* qconst, double* range) {
+    if (bytes < kHeaderBytes) return PFPL_ERR_CORRUPT;
+    if (h[0] != 'P' || h[1] != 'F' || h[2] != 'P' || h[3] != 'L' || h[4] != 1) return PFPL_ERR_CORRUPT;
+    if (h[5] > 1 || h[6] > 2 || (h[7] & ~3u)) return PFPL_ERR_CORRUPT;
+    uint64_t f[5];
+    for (int i = 0; i < 5; ++i) {
+        f[i] = 0;
+        for (int k = 7; k >= 0; --k) f[i] = (f[i] << 8) | h[8 + 8 * i + k];
+    }
+    if (f[4] != kChunkBytes) return PFPL_ERR_CORRUPT;    // chunk bytes + reserved 0
+    if (f[0] > (1ull << 40)) return PFPL_ERR_CORRUPT;
+    if (n) *n = f[0];
+    if (dtype) *dtype = h[5];
+    if (bound) *bound = h[6];
+    if (eps) *eps = u2d_h(f[1]);
+    if (flags) *flags = h[7];
+    if (qconst) *qconst = f[2];
+    if (range) *range = u2d_h(f[3]);
+    return PFPL_OK;
+}
+
+// decoder constants from the header (validated: corrupt constants -> error)
+int decode_qconst(int dtype, int bound, unsigned flags, uint64_t qk, QConst* qc, int* mode) {
+    memset(qc, 0, sizeof(*qc));
+    qc->flags = flags;
+    if (flags & HF_RAWWORDS) { *mode = MODE_RAW; return PFPL_OK; }
+    if (dtype == PFPL_F32) {
+        if (qk >> 32) return PFPL_ERR_CORRUPT;
+        const float c = u2f_h((uint32_t)qk);
+        if (bound == PFPL_REL) {
+            if (!(c > 0.0f) || std::isinf(c)) return PFPL_ERR_CORRUPT;
+            qc->b = f2u_h(c);
+            *mode = MODE_REL;
+        } else {
+            if (!(c >= FLT_MIN && c <= FLT_MAX / 2)) return PFPL_ERR_CORRUPT;
+            qc->a = f2u_h(c); qc->c = f2u_h(2.0f * c);
+            *mode = MODE_ABS;
+        }
+    } else {
+        const double c = u2d_h(qk);
+        if (bound == PFPL_REL) {
+            if (!(c > 0.0) || std::isinf(c)) return PFPL_ERR_CORRUPT;
+            qc->b = d2u_h(c);
+            *mode = MODE_REL;
+        } else {
+            if (!(c >= DBL_MIN && c <= DBL_MAX / 2)) return PFPL_ERR_CORRUPT;
+            qc->a = d2u_h(c); qc->c = d2u_h(2.0 * c);
+            *mode = MODE_ABS;
+        }
+    }
+    return PFPL_OK;
+}
+
+int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t first_chunk,
+                       uint64_t nchunks, const uint8_t* payload, uint64_t payload_bytes,
+                       void* out, uint64_t cap, int* err_dev, cudaStream_t s, uint64_t* n_out) {
+    uint64_t n = 0, qk = 0;
+    int dtype = 0, bound = 0;
+    unsigned flags = 0;
+    int st = parse_header(hdr, kHeaderBytes, &n, &dtype, &bound, nullptr, &flags, &qk, nullptr);
+    if (st != PFPL_OK) return st;
+    QConst qc;
+    int mode = 0;
+    st = decode_qconst(dtype, bound, flags, qk, &qc, &mode);
+    if (st != PFPL_OK) return st;
+    const uint64_t cw = kChunkBytes / tsz(dtype);
+    const uint64_t C = chunks_of(n, dtype);
+    if (first_chunk > C || nchunks > C - first_chunk) return PFPL_ERR_ARG;
+    const uint64_t e0 = first_chunk * cw;
+    const uint64_t nloc = nchunks ? ((first_chunk + nchunks) * cw < n ? nchunks * cw : n - e0) : 0;
+    if (n_out) *n_out = nloc;
+    if (cap < nloc * tsz(dtype)) return PFPL_ERR_CAPACITY;
+    if (!aligned16(out)) return PFPL_ERR_ALIGN;
+    if (nchunks == 0) return payload_bytes == 0 ? PFPL_OK : PFPL_ERR_CORRUPT;
+    Scratch* sc = nullptr;
+    st = get_scratch(s, nchunks, &sc);
+    if (st != PFPL_OK) return st;
+    DecParams p;
+    memset(&p, 0, sizeof(p));
+    p.in = payload;
+    p.in_bytes = payload_bytes;
+    p.table = table_dev;
+    p.n = nloc;
+    p.C = nchunks;
+    p.out = out;
+    p.status = sc->status;
+    p.ticket = sc->ticket;
+    p.ticket_base = sc->ticket_val;
+    p.epoch = sc->epoch;
+    p.qc = qc;
+    p.err = err_dev;
+    const bool ms = (flags & HF_MS) != 0;
+    const int grid = decode_grid(dtype, mode, ms, nchunks);
+    CK(launch_decode(dtype, mode, ms, p, grid, s));
+    g_launches += 1;
+    sc->ticket_val += nchunks + (uint64_t)grid;
+    return PFPL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+uint64_t pfpl_max_compressed_bytes(uint64_t n, int dtype) {
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return 0;
+    return kHeaderBytes + 4 * chunks_of(n, dtype) + n * tsz(dtype);
+}
+
+int pfpl_compress_async(const void* in, uint64_t n, int dtype, int bound, double eps,
+                        unsigned opts, void* out, uint64_t cap, uint64_t* result_dev,
+                        void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return PFPL_ERR_ARG;
+    const uint64_t C = chunks_of(n, dtype);
+    if (cap < kHeaderBytes + 4 * C) return PFPL_ERR_CAPACITY;
+    if (result_dev) CK(cudaMemsetAsync(result_dev, 0, 16, s));
+    return enqueue_compress(in, n, n, dtype, bound, eps, opts, nullptr, (uint8_t*)out, cap,
+                            (uint32_t*)((uint8_t*)out + kHeaderBytes), kHeaderBytes + 4 * C, 1,
+                            result_dev, s, nullptr);
+}
+
+int pfpl_compress_ex(const void* in, uint64_t n, int dtype, int bound, double eps, unsigned opts,
+                     void* out, uint64_t* out_bytes, void* stream) {
+    if (!out_bytes) return PFPL_ERR_ARG;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return PFPL_ERR_ARG;
+    const uint64_t C = chunks_of(n, dtype);
+    const uint64_t cap = *out_bytes;
+    if (cap < kHeaderBytes + 4 * C) return PFPL_ERR_CAPACITY;
+    Scratch* sc = nullptr;
+    int st = enqueue_compress(in, n, n, dtype, bound, eps, opts, nullptr, (uint8_t*)out, cap,
+                              (uint32_t*)((uint8_t*)out + kHeaderBytes), kHeaderBytes + 4 * C, 1,
+                              nullptr, s, &sc);
+    if (st != PFPL_OK) return st;
+    CK(cudaMemcpyAsync(sc->host, sc->result, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const uint64_t total = sc->host[0];
+    if (total > cap) return PFPL_ERR_CAPACITY;
+    *out_bytes = total;
+    return PFPL_OK;
+}
+
+int pfpl_compress(const void* in, uint64_t n, int dtype, int bound, double eps, void* out,
+                  uint64_t* out_bytes, void* stream) {
+    return pfpl_compress_ex(in, n, dtype, bound, eps, 0u, out, out_bytes, stream);
+}
+
+int pfpl_peek_header(const void* hdr, uint64_t bytes, uint64_t* n, int* dtype, int* bound,
+                     double* eps, unsigned* flags) {
+    if (!hdr) return PFPL_ERR_ARG;
+    return parse_header((const uint8_t*)hdr, bytes, n, dtype, bound, eps, flags, nullptr, nullptr);
+}
+
+int pfpl_decompress_async(const void* in, uint64_t in_bytes, const void* hdr_host, void* out,
+                          uint64_t cap, uint64_t* result_dev, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!in || !hdr_host || !result_dev) return PFPL_ERR_ARG;
+    if (!aligned16(in)) return PFPL_ERR_ALIGN;
+    uint64_t n = 0;
+    int dtype = 0;
+    int st = parse_header((const uint8_t*)hdr_host, kHeaderBytes, &n, &dtype, nullptr, nullptr,
+                          nullptr, nullptr, nullptr);
+    if (st != PFPL_OK) return st;
+    if (in_bytes < kHeaderBytes) return PFPL_ERR_CORRUPT;
+    const uint64_t C = chunks_of(n, dtype);
+    if (in_bytes < kHeaderBytes + 4 * C) return PFPL_ERR_CORRUPT;
+    CK(cudaMemsetAsync(result_dev, 0, 16, s));
+    const uint8_t* base = (const uint8_t*)in;
+    uint64_t nout = 0;
+    return enqueue_decompress((const uint8_t*)hdr_host, (const uint32_t*)(base + kHeaderBytes), 0,
+                              C, base + kHeaderBytes + 4 * C, in_bytes - kHeaderBytes - 4 * C, out,
+                              cap, (int*)(result_dev + 1), s, &nout);
+}
+
+int pfpl_decompress(const void* in, uint64_t in_bytes, void* out, uint64_t* out_bytes,
+                    void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!in || !out_bytes) return PFPL_ERR_ARG;
+    if (!aligned16(in)) return PFPL_ERR_ALIGN;
+    if (in_bytes < kHeaderBytes) return PFPL_ERR_CORRUPT;
+    Scratch* sc = nullptr;
+    int st = get_scratch(s, 0, &sc);
+    if (st != PFPL_OK) return st;
+    CK(cudaMemcpyAsync(sc->hdr_host, in, kHeaderBytes, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    uint8_t hdr[kHeaderBytes];
+    memcpy(hdr, sc->hdr_host, kHeaderBytes);
+    uint64_t n = 0;
+    int dtype = 0;
+    st = parse_header(hdr, kHeaderBytes, &n, &dtype, nullptr, nullptr, nullptr, nullptr, nullptr);
+    if (st != PFPL_OK) return st;
+    const uint64_t C = chunks_of(n, dtype);
+    if (in_bytes < kHeaderBytes + 4 * C) return PFPL_ERR_CORRUPT;
+    CK(cudaMemsetAsync(sc->result + 1, 0, 8, s));
+    const uint8_t* base = (const uint8_t*)in;
+    uint64_t nout = 0;
+    st = enqueue_decompress(hdr, (const uint32_t*)(base + kHeaderBytes), 0, C,
+                            base + kHeaderBytes + 4 * C, in_bytes - kHeaderBytes - 4 * C, out,
+                            *out_bytes, (int*)(sc->result + 1), s, &nout);
+    if (st != PFPL_OK) return st;
+    CK(cudaMemcpyAsync(sc->host + 1, sc->result + 1, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const int err = (int)(int32_t)(uint32_t)sc->host[1];
+    if (err) return err;
+    *out_bytes = nout * tsz(dtype);
+    return PFPL_OK;
+}
+
+int pfpl_minmax(const void* in, uint64_t n, int dtype, double* mnmx_dev, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return PFPL_ERR_ARG;
+    if ((n && !in) || !mnmx_dev) return PFPL_ERR_ARG;
+    if (!aligned16(in)) return PFPL_ERR_ALIGN;
+    Scratch* sc = nullptr;
+    int st = get_scratch(s, 0, &sc);
+    if (st != PFPL_OK) return st;
+    CK(launch_minmax(dtype, in, n, sc->partial, kMinmaxBlocks, s));
+    CK(launch_minmax_final(sc->partial, kMinmaxBlocks, mnmx_dev, s));
+    g_launches += 2;
+    return PFPL_OK;
+}
+
+int pfpl_compress_shard(const void* in, uint64_t n_local, uint64_t first_chunk, uint64_t n_total,
+                        int dtype, int bound, double eps, unsigned opts, const double* mnmx_dev,
+                        void* out, uint64_t cap, uint64_t* payload_bytes, void* hdr_out_host,
+                        void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return PFPL_ERR_ARG;
+    if (!payload_bytes) return PFPL_ERR_ARG;
+    const uint64_t cw = kChunkBytes / tsz(dtype);
+    const uint64_t Ct = chunks_of(n_total, dtype);
+    const uint64_t Cl = chunks_of(n_local, dtype);
+    if (first_chunk + Cl > Ct) return PFPL_ERR_ARG;
+    if (first_chunk * cw + n_local > n_total) return PFPL_ERR_ARG;
+    if (n_local % cw && first_chunk * cw + n_local != n_total) return PFPL_ERR_ARG;
+    if (bound == PFPL_NOA && !mnmx_dev) return PFPL_ERR_ARG;
+    if (cap < 4 * Cl) return PFPL_ERR_CAPACITY;
+    Scratch* sc = nullptr;
+    int st = enqueue_compress(in, n_local, n_total, dtype, bound, eps, opts, mnmx_dev,
+                              (uint8_t*)out, cap, (uint32_t*)out, 4 * Cl, 0, nullptr, s, &sc);
+    if (st != PFPL_OK) return st;
+    CK(cudaMemcpyAsync(sc->host, sc->result, 8, cudaMemcpyDeviceToHost, s));
+    QConst qc;
+    int mode = 0;
+    host_qconst(dtype, bound, eps, opts, &qc, &mode);
+    QConst qch;
+    if (bound == PFPL_NOA) CK(cudaMemcpyAsync(&qch, sc->qc_dev, sizeof(QConst), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (bound == PFPL_NOA) qc = qch;
+    const uint64_t total = sc->host[0];
+    if (total > cap) return PFPL_ERR_CAPACITY;
+    *payload_bytes = total - 4 * Cl;
+    if (hdr_out_host) {
+        uint8_t* h = (uint8_t*)hdr_out_host;
+        memset(h, 0, kHeaderBytes);
+        h[0] = 'P'; h[1] = 'F'; h[2] = 'P'; h[3] = 'L';
+        h[4] = 1; h[5] = (uint8_t)dtype; h[6] = (uint8_t)bound; h[7] = (uint8_t)qc.flags;
+        const uint64_t f[5] = {n_total, d2u_h(eps), qc.qconst, d2u_h(qc.range), (uint64_t)kChunkBytes};
+        for (int i = 0; i < 5; ++i)
+            for (int k = 0; k < 8; ++k) h[8 + 8 * i + k] = (uint8_t)(f[i] >> (8 * k));
+    }
+    return PFPL_OK;
+}
+
+int pfpl_decompress_chunks(const void* hdr_host, const uint32_t* table_host, uint64_t first_chunk,
+                           uint64_t n_chunks, const void* payload, uint64_t payload_bytes,
+                           void* out, uint64_t cap, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!hdr_host || (n_chunks && (!table_host || !payload))) return PFPL_ERR_ARG;
+    if (payload && !aligned16(payload)) return PFPL_ERR_ALIGN;
+    Scratch* sc = nullptr;
+    int st = get_scratch(s, n_chunks, &sc);
+    if (st != PFPL_OK) return st;
+    if (n_chunks > sc->table_cap) {
+        if (sc->table_dev) CK(cudaFree(sc->table_dev));
+        CK(cudaMalloc(&sc->table_dev, n_chunks * 4));
+        sc->table_cap = n_chunks;
+    }
+    if (n_chunks) CK(cudaMemcpyAsync(sc->table_dev, table_host, n_chunks * 4, cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(sc->result + 1, 0, 8, s));
+    uint64_t nout = 0;
+    st = enqueue_decompress((const uint8_t*)hdr_host, sc->table_dev, first_chunk, n_chunks,
+                            (const uint8_t*)payload, payload_bytes, out, cap, (int*)(sc->result + 1),
+                            s, &nout);
+    if (st != PFPL_OK) return st;
+    CK(cudaMemcpyAsync(sc->host + 1, sc->result + 1, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const int err = (int)(int32_t)(uint32_t)sc->host[1];
+    return err ? err : PFPL_OK;
+}
+
+const char* pfpl_strerror(int st) {
+    switch (st) {
+        case PFPL_OK: return "ok";
+        case PFPL_ERR_ARG: return "invalid argument";
+        case PFPL_ERR_BOUND: return "invalid error bound";
+        case PFPL_ERR_CAPACITY: return "output capacity too small";
+        case PFPL_ERR_CORRUPT: return "corrupt stream";
+        case PFPL_ERR_ALIGN: return "buffer not 16-byte aligned";
+        case PFPL_ERR_CUDA: return "CUDA runtime error";
+        default: return "unknown status";
+    }
+}
+
+int pfpl_last_cuda_error(void) { return g_last_cuda.load(); }
+
+int pfpl_release_scratch(void) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    for (auto it = g_scratch.begin(); it != g_scratch.end();) {
+        if (it->first.first != dev) { ++it; continue; }
+        Scratch* sc = it->second;
+        cudaDeviceSynchronize();
+        cudaFree(sc->status); cudaFree(sc->ticket); cudaFree(sc->qc_dev); cudaFree(sc->mnmx);
+        cudaFree(sc->partial); cudaFree(sc->result); cudaFreeHost(sc->host);
+        cudaFreeHost(sc->hdr_host); cudaFree(sc->table_dev);
+        delete sc;
+        it = g_scratch.erase(it);
+    }
+    return PFPL_OK;
+}
+
+uint64_t pfpl_launch_count(void) { return g_launches.load(); }
+
+const char* pfpl_version(void) { return "pfpl-b200 1.0 sm_100a (stream format v1)"; }
+
+}  // extern "C"

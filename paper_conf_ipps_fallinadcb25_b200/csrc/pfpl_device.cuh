@@ -1,0 +1,390 @@
+// pfpl_device.cuh -- sm_100a device building blocks of the PFPL hot path.
+//
+// Quantizers, portable log2/pow2 (reading R5), bit-plane
+// transposes, warp/block scans and look-back
+// (Merrill & Garland).  Compiled with -fmad=false, IEEE division and
+// no FTZ, so every floating-point operation is one correctly rounded IEEE
+// operation, as P:110 requires for CPU/GPU bit-identity.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "pfpl_internal.h"
+
+namespace pfpl {
+
+#define PFPL_FULL 0xFFFFFFFFu
+#define PFPL_HD __host__ __device__ __forceinline__
+
+// ------------------------------------------------------------------------
+// traits: one thread owns 32 consecutive elements; a chunk is 16384 bytes
+// ------------------------------------------------------------------------
+template <typename T> struct Tr;
+template <> struct Tr<float> {
+    typedef uint32_t W;
+    static constexpr int B = 32, CW = 4096, NT = 128, NW = 4, S = 4, MANT = 23;
+};
+template <> struct Tr<double> {
+    typedef uint64_t W;
+    static constexpr int B = 64, CW = 2048, NT = 64, NW = 2, S = 8, MANT = 52;
+};
+
+PFPL_HD uint32_t f2u(float x) { union { float f; uint32_t u; } v; v.f = x; return v.u; }
+PFPL_HD float u2f(uint32_t x) { union { float f; uint32_t u; } v; v.u = x; return v.f; }
+PFPL_HD uint64_t d2u(double x) { union { double f; uint64_t u; } v; v.f = x; return v.u; }
+PFPL_HD double u2d(uint64_t x) { union { double f; uint64_t u; } v; v.u = x; return v.f; }
+
+// ------------------------------------------------------------------------
+// portable log2 / pow2.  Format-version-1 constants: nearest binary32 /
+// binary64 to 2/(k ln 2) (atanh series of log2) and ln2^j/j! (Taylor of 2^f).
+// Plain operators: -fmad=false (device) / -ffp-contract=off (host) keep every
+// operation separately rounded.
+// ------------------------------------------------------------------------
+PFPL_HD float log2p_f32(float a) {
+    uint32_t u = f2u(a);
+    int e = (int)((u >> 23) & 0xFFu) - 127;
+    float m = u2f((u & 0x007FFFFFu) | 0x3F800000u);
+    if (m > u2f(0x3FB504F3u)) { m = m * 0.5f; e = e + 1; }
+    float t = (m - 1.0f) / (m + 1.0f);
+    float t2 = t * t;
+    float p = u2f(0x3ED30BB1u);
+    p = p * t2; p = p + u2f(0x3F13BB63u);
+    p = p * t2; p = p + u2f(0x3F76384Fu);
+    p = p * t2; p = p + u2f(0x4038AA3Bu);
+    float r = t * p;
+    return (float)e + r;
+}
+
+PFPL_HD float pow2p_f32(float y) {
+    float k = rintf(y);
+    float f = y - k;
+    float p = u2f(0x377FE5FEu);
+    p = p * f; p = p + u2f(0x39218489u);
+    p = p * f; p = p + u2f(0x3AAEC3FFu);
+    p = p * f; p = p + u2f(0x3C1D955Bu);
+    p = p * f; p = p + u2f(0x3D635847u);
+    p = p * f; p = p + u2f(0x3E75FDF0u);
+    p = p * f; p = p + u2f(0x3F317218u);
+    p = p * f; p = p + 1.0f;
+    if (!(k <= 127.0f)) return u2f(0x7F800000u);
+    if (k < -126.0f) return 0.0f;
+    int ki = (int)k;
+    return p * u2f((uint32_t)(ki + 127) << 23);
+}
+
+PFPL_HD double log2p_f64(double a) {
+    uint64_t u = d2u(a);
+    int e = (int)((u >> 52) & 0x7FFu) - 1023;
+    double m = u2d((u & 0x000FFFFFFFFFFFFFull) | 0x3FF0000000000000ull);
+    if (m > u2d(0x3FF6A09E667F3BCDull)) { m = m * 0.5; e = e + 1; }
+    double t = (m - 1.0) / (m + 1.0);
+    double t2 = t * t;
+    double p = u2d(0x3FC1964EC6FC9491ull);                         // c21
+    p = p * t2; p = p + u2d(0x3FC3703C1F4D0FFEull);                 // c19
+    p = p * t2; p = p + u2d(0x3FC5B9AC9B743F0Dull);                 // c17
+    p = p * t2; p = p + u2d(0x3FC89F3B1694CFFEull);                 // c15
+    p = p * t2; p = p + u2d(0x3FCC68F568D31760ull);                 // c13
+    p = p * t2; p = p + u2d(0x3FD0C9A84994022Dull);                 // c11
+    p = p * t2; p = p + u2d(0x3FD484B13D7C02A9ull);                 // c9
+    p = p * t2; p = p + u2d(0x3FDA61762A7ADED9ull);                 // c7
+    p = p * t2; p = p + u2d(0x3FE2776C50EF9BFEull);                 // c5
+    p = p * t2; p = p + u2d(0x3FEEC709DC3A03FDull);                 // c3
+    p = p * t2; p = p + u2d(0x40071547652B82FEull);                 // c1
+    double r = t * p;
+    return (double)e + r;
+}
+
+PFPL_HD double pow2p_f64(double y) {
+    double k = rint(y);
+    double f = y - k;
+    double p = u2d(0x3D7816193166D0F9ull);                          // ln2^13/13!
+    p = p * f; p = p + u2d(0x3DBC3BD650FC2986ull);
+    p = p * f; p = p + u2d(0x3DFE8CAC7351BB25ull);
+    p = p * f; p = p + u2d(0x3E3E4CF5158B8ECAull);
+    p = p * f; p = p + u2d(0x3E7B5253D395E7C4ull);
+    p = p * f; p = p + u2d(0x3EB62C0223A5C824ull);
+    p = p * f; p = p + u2d(0x3EEFFCBFC588B0C7ull);
+    p = p * f; p = p + u2d(0x3F2430912F86C787ull);
+    p = p * f; p = p + u2d(0x3F55D87FE78A6731ull);
+    p = p * f; p = p + u2d(0x3F83B2AB6FBA4E77ull);
+    p = p * f; p = p + u2d(0x3FAC6B08D704A0C0ull);
+    p = p * f; p = p + u2d(0x3FCEBFBDFF82C58Full);
+    p = p * f; p = p + u2d(0x3FE62E42FEFA39EFull);
+    p = p * f; p = p + 1.0;
+    if (!(k <= 1023.0)) return u2d(0x7FF0000000000000ull);
+    if (k < -1022.0) return 0.0;
+    long long ki = (long long)k;
+    return p * u2d((uint64_t)(ki + 1023) << 52);
+}
+
+// ------------------------------------------------------------------------
+// quantizers: value -> word (bin code or raw bits)
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t zz(int32_t b) { return ((uint32_t)b << 1) ^ (uint32_t)(b >> 31); }
+__device__ __forceinline__ uint64_t zz(int64_t b) { return ((uint64_t)b << 1) ^ (uint64_t)(b >> 63); }
+__device__ __forceinline__ int32_t unzz(uint32_t z) { return (int32_t)((z >> 1) ^ (0u - (z & 1u))); }
+__device__ __forceinline__ int64_t unzz(uint64_t z) { return (int64_t)((z >> 1) ^ (0ull - (z & 1ull))); }
+
+template <typename T> struct QF;
+template <> struct QF<float> {
+    float a, b, c;
+    __device__ __forceinline__ void load(const QConst& q) { a = u2f((uint32_t)q.a); b = u2f((uint32_t)q.b); c = u2f((uint32_t)q.c); }
+    // ABS/NOA: a = eps_eff, b = inv, c = eb2.  Bin = rint(v*inv); decode
+    // immediately and keep the bin only if |v - bin*2eps| <= eps (R7);
+    // |bin| < 2^22 so the zigzag code stays in the denormal range (R8).
+    __device__ __forceinline__ uint32_t abs_q(float v) const {
+        float s = v * b;
+        float rb = rintf(s);
+        bool ok = fabsf(rb) < 4194304.0f;
+        float vr = rb * c;
+        float diff = fabsf(v - vr);
+        ok = ok && (diff <= a);
+        int32_t bi = __float2int_rz(rb);
+        return ok ? zz(bi) : f2u(v);
+    }
+    __device__ __forceinline__ float abs_dq(uint32_t w) const {
+        return w < 0x00800000u ? __int2float_rn(unzz(w)) * c : u2f(w);
+    }
+    // REL: a = c_lo, b = w, c = inv_w.  log-space bin (R5), conservative
+    // 1-ulp-shrunk check (R7), sign+bin in the negative-NaN payload (R10),
+    // sign and exponent bits of every word inverted (R11).
+    __device__ __forceinline__ uint32_t rel_q(float v) const {
+        uint32_t u = f2u(v);
+        uint32_t sign = u >> 31;
+        uint32_t au = u & 0x7FFFFFFFu;
+        uint32_t q0 = au > 0x7F800000u ? au : u;
+        if (au >= 0x00800000u && au < 0x7F800000u) {
+            float av = u2f(au);
+            float L = log2p_f32(av);
+            float s = L * c;
+            float rb = rintf(s);
+            if (fabsf(rb) < 2097152.0f) {
+                float y = rb * b;
+                float r = pow2p_f32(y);
+                float lo = u2f(f2u(av / a) + 1u);
+                float hi = u2f(f2u(av * a) - 1u);
+                if (lo <= r && r <= hi)
+                    q0 = 0xFF800000u | (1u + ((zz(__float2int_rz(rb)) << 1) | sign));
+            }
+        }
+        return q0 ^ 0xFF800000u;
+    }
+    __device__ __forceinline__ float rel_dq(uint32_t w) const {
+        uint32_t u = w ^ 0xFF800000u;
+        if ((u & 0xFF800000u) == 0xFF800000u && (u & 0x007FFFFFu) != 0) {
+            uint32_t t = (u & 0x007FFFFFu) - 1u;
+            float mag = pow2p_f32(__int2float_rn(unzz(t >> 1)) * b);
+            return (t & 1u) ? -mag : mag;
+        }
+        return u2f(u);
+    }
+};
+template <> struct QF<double> {
+    double a, b, c;
+    __device__ __forceinline__ void load(const QConst& q) { a = u2d(q.a); b = u2d(q.b); c = u2d(q.c); }
+    __device__ __forceinline__ uint64_t abs_q(double v) const {
+        double s = v * b;
+        double rb = rint(s);
+        bool ok = fabs(rb) < 2251799813685248.0;
+        double vr = rb * c;
+        double diff = fabs(v - vr);
+        ok = ok && (diff <= a);
+        int64_t bi = (int64_t)__double2ll_rz(rb);
+        return ok ? zz(bi) : d2u(v);
+    }
+    __device__ __forceinline__ double abs_dq(uint64_t w) const {
+        return w < 0x0010000000000000ull ? __ll2double_rn((long long)unzz(w)) * c : u2d(w);
+    }
+    __device__ __forceinline__ uint64_t rel_q(double v) const {
+        uint64_t u = d2u(v);
+        uint64_t sign = u >> 63;
+        uint64_t au = u & 0x7FFFFFFFFFFFFFFFull;
+        uint64_t q0 = au > 0x7FF0000000000000ull ? au : u;
+        if (au >= 0x0010000000000000ull && au < 0x7FF0000000000000ull) {
+            double av = u2d(au);
+            double L = log2p_f64(av);
+            double s = L * c;
+            double rb = rint(s);
+            if (fabs(rb) < 1125899906842624.0) {
+                double y = rb * b;
+                double r = pow2p_f64(y);
+                double lo = u2d(d2u(av / a) + 1u);
+                double hi = u2d(d2u(av * a) - 1u);
+                if (lo <= r && r <= hi)
+                    q0 = 0xFFF0000000000000ull | (1ull + ((zz((int64_t)__double2ll_rz(rb)) << 1) | sign));
+            }
+        }
+        return q0 ^ 0xFFF0000000000000ull;
+    }
+    __device__ __forceinline__ double rel_dq(uint64_t w) const {
+        uint64_t u = w ^ 0xFFF0000000000000ull;
+        if ((u & 0xFFF0000000000000ull) == 0xFFF0000000000000ull &&
+            (u & 0x000FFFFFFFFFFFFFull) != 0) {
+            uint64_t t = (u & 0x000FFFFFFFFFFFFFull) - 1u;
+            double mag = pow2p_f64(__ll2double_rn((long long)unzz(t >> 1)) * b);
+            return (t & 1u) ? -mag : mag;
+        }
+        return u2d(u);
+    }
+};
+
+template <typename T, int MODE>
+__device__ __forceinline__ typename Tr<T>::W quantize(const QF<T>& q, T v, bool raw) {
+    if (MODE == MODE_RAW) return sizeof(T) == 4 ? (typename Tr<T>::W)f2u((float)v) : (typename Tr<T>::W)d2u((double)v);
+    if (MODE == MODE_NOA && raw) {
+        if (sizeof(T) == 4) return (typename Tr<T>::W)f2u((float)v);
+        return (typename Tr<T>::W)d2u((double)v);
+    }
+    if (MODE == MODE_REL) return q.rel_q(v);
+    return q.abs_q(v);
+}
+
+template <typename T, int MODE>
+__device__ __forceinline__ T dequantize(const QF<T>& q, typename Tr<T>::W w, bool raw);
+template <> __device__ __forceinline__ float dequantize<float, MODE_ABS>(const QF<float>& q, uint32_t w, bool) { return q.abs_dq(w); }
+template <> __device__ __forceinline__ float dequantize<float, MODE_NOA>(const QF<float>& q, uint32_t w, bool raw) { return raw ? u2f(w) : q.abs_dq(w); }
+template <> __device__ __forceinline__ float dequantize<float, MODE_REL>(const QF<float>& q, uint32_t w, bool) { return q.rel_dq(w); }
+template <> __device__ __forceinline__ float dequantize<float, MODE_RAW>(const QF<float>&, uint32_t w, bool) { return u2f(w); }
+template <> __device__ __forceinline__ double dequantize<double, MODE_ABS>(const QF<double>& q, uint64_t w, bool) { return q.abs_dq(w); }
+template <> __device__ __forceinline__ double dequantize<double, MODE_NOA>(const QF<double>& q, uint64_t w, bool raw) { return raw ? u2d(w) : q.abs_dq(w); }
+template <> __device__ __forceinline__ double dequantize<double, MODE_REL>(const QF<double>& q, uint64_t w, bool) { return q.rel_dq(w); }
+template <> __device__ __forceinline__ double dequantize<double, MODE_RAW>(const QF<double>&, uint64_t w, bool) { return u2d(w); }
+
+// ------------------------------------------------------------------------
+// residual codes: negabinary (default) or zigzag (flag A1)
+// ------------------------------------------------------------------------
+template <bool MS> __device__ __forceinline__ uint32_t rcode(uint32_t d) {
+    return MS ? ((d << 1) ^ (uint32_t)((int32_t)d >> 31)) : ((d + 0xAAAAAAAAu) ^ 0xAAAAAAAAu);
+}
+template <bool MS> __device__ __forceinline__ uint64_t rcode(uint64_t d) {
+    return MS ? ((d << 1) ^ (uint64_t)((int64_t)d >> 63))
+              : ((d + 0xAAAAAAAAAAAAAAAAull) ^ 0xAAAAAAAAAAAAAAAAull);
+}
+template <bool MS> __device__ __forceinline__ uint32_t rdecode(uint32_t r) {
+    return MS ? ((r >> 1) ^ (0u - (r & 1u))) : ((r ^ 0xAAAAAAAAu) - 0xAAAAAAAAu);
+}
+template <bool MS> __device__ __forceinline__ uint64_t rdecode(uint64_t r) {
+    return MS ? ((r >> 1) ^ (0ull - (r & 1ull)))
+              : ((r ^ 0xAAAAAAAAAAAAAAAAull) - 0xAAAAAAAAAAAAAAAAull);
+}
+
+// ------------------------------------------------------------------------
+// bit-plane transpose of 32 words with values < 2^K (K in {4,8,16,32}):
+// out[b] bit j = bit b of in[j].  Pack 32/K elements per word (element j at
+// word j%K, position K*(j/K)+bit), then exchange word-index bit i with
+// position bit i for i < log2 K (delta swaps).  The exchanges are involutions,
+// so the inverse is: same exchanges, then unpack.
+// ------------------------------------------------------------------------
+template <int I> __device__ __forceinline__ void xchg(uint32_t& a, uint32_t& b) {
+    if (I == 4) {
+        uint32_t na = __byte_perm(a, b, 0x5410), nb = __byte_perm(a, b, 0x7632);
+        a = na; b = nb;
+    } else if (I == 3) {
+        uint32_t na = __byte_perm(a, b, 0x6240), nb = __byte_perm(a, b, 0x7351);
+        a = na; b = nb;
+    } else {
+        constexpr uint32_t M = I == 0 ? 0x55555555u : I == 1 ? 0x33333333u : 0x0F0F0F0Fu;
+        constexpr int s = 1 << I;
+        uint32_t t = ((a >> s) ^ b) & M;
+        b ^= t;
+        a ^= t << s;
+    }
+}
+
+template <int K> __device__ __forceinline__ void xchg_all(uint32_t (&o)[K]) {
+#pragma unroll
+    for (int i = 0; (1 << i) < K; ++i) {
+#pragma unroll
+        for (int a = 0; a < K; ++a) {
+            if (a & (1 << i)) continue;
+            const int b = a | (1 << i);
+            switch (i) {
+                case 0: xchg<0>(o[a], o[b]); break;
+                case 1: xchg<1>(o[a], o[b]); break;
+                case 2: xchg<2>(o[a], o[b]); break;
+                case 3: xchg<3>(o[a], o[b]); break;
+                default: xchg<4>(o[a], o[b]); break;
+            }
+        }
+    }
+}
+
+template <int K> __device__ __forceinline__ void transpose_fwd(const uint32_t (&in)[32], uint32_t (&o)[K]) {
+    constexpr int H = 32 / K;
+#pragma unroll
+    for (int w = 0; w < K; ++w) {
+        uint32_t x = in[w];
+#pragma unroll
+        for (int h = 1; h < H; ++h) x |= in[w + K * h] << (K * h);
+        o[w] = x;
+    }
+    xchg_all<K>(o);
+}
+
+template <int K> __device__ __forceinline__ void transpose_inv(uint32_t (&o)[K], uint32_t (&out)[32]) {
+    constexpr int H = 32 / K;
+    xchg_all<K>(o);
+#pragma unroll
+    for (int w = 0; w < K; ++w) {
+#pragma unroll
+        for (int h = 0; h < H; ++h)
+            out[w + K * h] = K == 32 ? o[w] : ((o[w] >> (K * h)) & ((1u << (K & 31)) - 1u));
+    }
+}
+
+// ------------------------------------------------------------------------
+// byte helpers
+// ------------------------------------------------------------------------
+// 0x01 in every non-zero byte of x
+__device__ __forceinline__ uint32_t nzbytes(uint32_t x) {
+    return (((x & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | x) >> 7 & 0x01010101u;
+}
+// gather the low bits of the 4 bytes of h (values 0/1) into a nibble
+__device__ __forceinline__ uint32_t nib(uint32_t h) { return (h * 0x10204080u) >> 28; }
+
+// ------------------------------------------------------------------------
+// scans
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int lane) {
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        uint32_t t = __shfl_up_sync(PFPL_FULL, v, d);
+        if (lane >= d) v += t;
+    }
+    return v;
+}
+__device__ __forceinline__ uint64_t warp_incl_scan64(uint64_t v, int lane) {
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        uint64_t t = __shfl_up_sync(PFPL_FULL, v, d);
+        if (lane >= d) v += t;
+    }
+    return v;
+}
+__device__ __forceinline__ uint64_t warp_sum64(uint64_t v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(PFPL_FULL, v, d);
+    return v;
+}
+
+// ------------------------------------------------------------------------
+// look-back descriptors: [63:48] epoch | [47:46] flag | [45:0] value
+// ------------------------------------------------------------------------
+constexpr uint64_t LB_A = 1, LB_P = 2;
+constexpr uint64_t LB_VAL = (1ull << 46) - 1;
+
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint4 ldg_nc_v4(const void* p) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+
+}  // namespace pfpl

@@ -1,0 +1,85 @@
+// pfpl_internal.h -- structures shared by the host API and the sm_100a kernels
+// of libpfpl.so.  Product code only; shares nothing with the CPU test reference.
+// Stream format and readings: DESIGN.md sections 3 and 5.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace pfpl {
+
+constexpr uint32_t kChunkBytes = 16384;   // P:141 "16 kB chunks" (R19: 16384 for both dtypes)
+constexpr uint32_t kHeaderBytes = 48;     // R18
+constexpr int kEPT = 32;                  // elements per thread (one 32-bit plane word)
+
+enum Mode : int { MODE_ABS = 0, MODE_REL = 1, MODE_RAW = 2, MODE_NOA = 3 };
+enum HdrFlags : uint32_t { HF_RAWWORDS = 1, HF_MS = 2 };
+
+// Quantizer constants.  Bit patterns of T values (f32 in the low 32 bits).
+//   ABS/NOA: a = eps_eff, b = inv = 0.5/eps_eff, c = eb2 = 2*eps_eff
+//   REL    : a = c_lo (largest T <= 1+eps), b = w = 2*log2p(c_lo), c = inv_w = 0.5/log2p(c_lo)
+struct QConst {
+    uint64_t a, b, c;
+    uint64_t qconst;   // header offset 24
+    double range;      // header offset 32 (NOA)
+    uint32_t flags;    // header byte 7
+    uint32_t pad;
+};
+
+struct EncParams {
+    const void* in;          // local elements (16B aligned)
+    uint64_t n;              // local element count
+    uint64_t C;              // local chunk count
+    uint8_t* out;            // stream base
+    uint64_t cap;            // capacity of out (bytes)
+    uint32_t* table;         // size table (local slice)
+    uint64_t payload_off;    // payload start relative to out
+    unsigned long long* status;   // look-back descriptors [C]
+    unsigned long long* ticket;   // monotone ticket counter
+    uint64_t ticket_base;
+    uint32_t epoch;
+    int write_header;
+    QConst qc;               // ABS/REL/RAW constants
+    const QConst* qc_dev;    // NOA: constants derived on the device
+    uint64_t* result;        // result[0] = stream bytes (payload_off + payload)
+    uint64_t n_total;        // header n
+    double eps;              // header eps
+    uint32_t dtype, bound;   // header bytes 5, 6
+};
+
+struct DecParams {
+    const uint8_t* in;       // payload base (first chunk's payload)
+    uint64_t in_bytes;       // bytes available from `in`
+    const uint32_t* table;   // size table (device)
+    uint64_t n;              // elements to produce
+    uint64_t C;              // chunks
+    void* out;
+    unsigned long long* status;
+    unsigned long long* ticket;
+    uint64_t ticket_base;
+    uint32_t epoch;
+    QConst qc;               // a/b/c as in QConst; decoder uses eb2 (ABS/NOA) or w (REL)
+    int* err;                // set to PFPL_ERR_CORRUPT on malformed chunks
+};
+
+// kernel launchers (pfpl_kernels.cu)
+cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int grid,
+                          cudaStream_t s);
+cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
+                          cudaStream_t s);
+cudaError_t launch_minmax(int dtype, const void* in, uint64_t n, double* partial,
+                          int blocks, cudaStream_t s);
+cudaError_t launch_minmax_final(const double* partial, int blocks, double* mnmx,
+                                cudaStream_t s);
+cudaError_t launch_noa_derive(int dtype, const double* mnmx, double eps, uint32_t ms_flag,
+                              QConst* qc_out, cudaStream_t s);
+cudaError_t launch_header_only(uint8_t* out, uint64_t n, int dtype, int bound, double eps,
+                               const QConst qc, const QConst* qc_dev, uint64_t* result,
+                               cudaStream_t s);
+int encode_grid(int dtype, int mode, bool ms, uint64_t C);
+int decode_grid(int dtype, int mode, bool ms, uint64_t C);
+
+// host-side portable log2 (same operation sequence as the device code)
+float log2p_host_f32(float a);
+double log2p_host_f64(double a);
+
+}  // namespace pfpl

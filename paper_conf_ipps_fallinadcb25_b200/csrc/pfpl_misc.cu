@@ -1,0 +1,156 @@
+// pfpl_misc.cu -- NOA min/max reduction, device-side
+// derivation of the NOA quantizer constants (reading R3/R4), header-only streams.
+#include <cfloat>
+#include "pfpl_device.cuh"
+
+namespace pfpl {
+
+constexpr int MM_THREADS = 256;
+
+__device__ __forceinline__ void mm_acc(double v, double& mn, double& mx) {
+    if (isfinite(v)) {                 // R2: finite values only
+        if (v == 0.0) v = 0.0;         // canonical +0
+        mn = v < mn ? v : mn;
+        mx = v > mx ? v : mx;
+    }
+}
+
+__device__ __forceinline__ void block_minmax(double& mn, double& mx, double* out2) {
+    __shared__ double smn[MM_THREADS / 32], smx[MM_THREADS / 32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+        const double a = __shfl_xor_sync(PFPL_FULL, mn, d), b = __shfl_xor_sync(PFPL_FULL, mx, d);
+        mn = a < mn ? a : mn;
+        mx = b > mx ? b : mx;
+    }
+    if (lane == 0) { smn[warp] = mn; smx[warp] = mx; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < MM_THREADS / 32; ++w) {
+            mn = smn[w] < mn ? smn[w] : mn;
+            mx = smx[w] > mx ? smx[w] : mx;
+        }
+        out2[0] = mn;
+        out2[1] = mx;
+    }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(MM_THREADS) minmax_kernel(const T* in, uint64_t n, double* partial) {
+    double mn = u2d(0x7FF0000000000000ull), mx = -mn;
+    constexpr int V = 16 / sizeof(T);
+    const uint64_t nv = n / V;
+    const uint64_t stride = (uint64_t)gridDim.x * MM_THREADS;
+    for (uint64_t i = (uint64_t)blockIdx.x * MM_THREADS + threadIdx.x; i < nv; i += stride) {
+        const uint4 v = ldg_nc_v4(in + i * V);
+        T x[V];
+        memcpy(x, &v, 16);
+#pragma unroll
+        for (int k = 0; k < V; ++k) mm_acc((double)x[k], mn, mx);
+    }
+    for (uint64_t i = nv * V + (uint64_t)blockIdx.x * MM_THREADS + threadIdx.x; i < n; i += stride)
+        mm_acc((double)in[i], mn, mx);
+    block_minmax(mn, mx, partial + 2 * blockIdx.x);
+}
+
+__global__ void __launch_bounds__(MM_THREADS) minmax_final_kernel(const double* partial, int blocks,
+                                                                  double* mnmx) {
+    double mn = u2d(0x7FF0000000000000ull), mx = -mn;
+    for (int i = threadIdx.x; i < blocks; i += MM_THREADS) {
+        const double a = partial[2 * i], b = partial[2 * i + 1];
+        mn = a < mn ? a : mn;
+        mx = b > mx ? b : mx;
+    }
+    block_minmax(mn, mx, mnmx);
+}
+
+// NOA constants (abs = eps * (max - min); R3: two round-downs so the
+// derived bound never exceeds the exact product; R1: largest T <= it; R4:
+// degenerate -> raw-words mode).  One thread.
+__global__ void noa_derive_kernel(int dtype, const double* mnmx, double eps, uint32_t ms_flag,
+                                  QConst* out) {
+    const double mn = mnmx[0], mx = mnmx[1];
+    const bool have = mn <= mx;
+    const double d = have ? mx - mn : 0.0;
+    const double r_lo = d > 0.0 ? u2d(d2u(d) - 1u) : 0.0;
+    const double e = eps * r_lo;
+    const double eps_abs = e > 0.0 ? u2d(d2u(e) - 1u) : 0.0;
+    QConst qc;
+    qc.a = qc.b = qc.c = qc.qconst = 0;
+    qc.range = d;
+    qc.flags = ms_flag;
+    qc.pad = 0;
+    if (dtype == 0) {
+        float ee = 0.0f;
+        if (eps_abs > 0.0) {
+            ee = __double2float_rn(eps_abs);
+            if (isinf(ee)) ee = FLT_MAX;
+            if ((double)ee > eps_abs) ee = u2f(f2u(ee) - 1u);
+        }
+        if (ee > FLT_MAX / 2) ee = FLT_MAX / 2;
+        if (!(ee >= FLT_MIN)) {
+            qc.flags |= HF_RAWWORDS;
+        } else {
+            qc.a = f2u(ee);
+            qc.b = f2u(0.5f / ee);
+            qc.c = f2u(2.0f * ee);
+            qc.qconst = f2u(ee);
+        }
+    } else {
+        double ee = eps_abs;
+        if (ee > DBL_MAX / 2) ee = DBL_MAX / 2;
+        if (!(ee >= DBL_MIN)) {
+            qc.flags |= HF_RAWWORDS;
+        } else {
+            qc.a = d2u(ee);
+            qc.b = d2u(0.5 / ee);
+            qc.c = d2u(2.0 * ee);
+            qc.qconst = d2u(ee);
+        }
+    }
+    *out = qc;
+}
+
+__global__ void header_only_kernel(uint8_t* out, uint64_t n, int dtype, int bound, double eps,
+                                   QConst qc, const QConst* qc_dev, uint64_t* result) {
+    if (qc_dev) qc = *qc_dev;
+    uint8_t h[48];
+    h[0] = 'P'; h[1] = 'F'; h[2] = 'P'; h[3] = 'L';
+    h[4] = 1; h[5] = (uint8_t)dtype; h[6] = (uint8_t)bound; h[7] = (uint8_t)qc.flags;
+    const uint64_t f[5] = {n, d2u(eps), qc.qconst, d2u(qc.range), (uint64_t)kChunkBytes};
+    for (int i = 0; i < 5; ++i)
+        for (int k = 0; k < 8; ++k) h[8 + 8 * i + k] = (uint8_t)(f[i] >> (8 * k));
+    for (int i = 0; i < 48; ++i) out[i] = h[i];
+    result[0] = 48;
+}
+
+cudaError_t launch_minmax(int dtype, const void* in, uint64_t n, double* partial, int blocks,
+                          cudaStream_t s) {
+    if (dtype == 0) minmax_kernel<float><<<blocks, MM_THREADS, 0, s>>>((const float*)in, n, partial);
+    else minmax_kernel<double><<<blocks, MM_THREADS, 0, s>>>((const double*)in, n, partial);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_minmax_final(const double* partial, int blocks, double* mnmx, cudaStream_t s) {
+    minmax_final_kernel<<<1, MM_THREADS, 0, s>>>(partial, blocks, mnmx);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_noa_derive(int dtype, const double* mnmx, double eps, uint32_t ms_flag,
+                              QConst* qc_out, cudaStream_t s) {
+    noa_derive_kernel<<<1, 1, 0, s>>>(dtype, mnmx, eps, ms_flag, qc_out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_header_only(uint8_t* out, uint64_t n, int dtype, int bound, double eps,
+                               const QConst qc, const QConst* qc_dev, uint64_t* result,
+                               cudaStream_t s) {
+    header_only_kernel<<<1, 1, 0, s>>>(out, n, dtype, bound, eps, qc, qc_dev, result);
+    return cudaGetLastError();
+}
+
+float log2p_host_f32(float a) { return log2p_f32(a); }
+double log2p_host_f64(double a) { return log2p_f64(a); }
+
+}  // namespace pfpl

@@ -1,0 +1,176 @@
+"""GPU <-> oracle parity through the C ABI (bit-for-bit identical
+compressed and decompressed output on CPUs and GPUs).
+
+Three checks per case: (1) GPU stream bytes == oracle stream bytes; (2) the
+GPU decodes the oracle's stream to the oracle's values, bit for bit; (3)
+every decoded value satisfies its bound exactly (tests/boundcheck.py).
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from tests.boundcheck import violations
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def pk():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_fallinadcb25_b200 as pk
+    return pk
+
+
+def _bits(a: np.ndarray):
+    return a.view(np.uint32 if a.dtype == np.float32 else np.uint64)
+
+
+def _check(pk, orc, x: np.ndarray, bound: str, eps: float, ms: bool = False):
+    xd = torch.from_numpy(x).cuda()
+    s_gpu = pk.compress(xd, bound, eps, ms=ms).cpu().numpy().tobytes()
+    s_cpu = orc.compress(x, bound, eps, ms=ms)
+    if s_gpu != s_cpu:
+        a, b = np.frombuffer(s_gpu, np.uint8), np.frombuffer(s_cpu, np.uint8)
+        k = min(a.size, b.size)
+        first = int(np.flatnonzero(a[:k] != b[:k])[0]) if np.any(a[:k] != b[:k]) else k
+        raise AssertionError(f"stream mismatch ({bound}, {x.dtype}, n={x.size}): "
+                             f"len gpu={len(s_gpu)} cpu={len(s_cpu)} first diff at byte {first}")
+    y_cpu = orc.decompress(s_cpu)
+    buf = torch.frombuffer(bytearray(s_cpu), dtype=torch.uint8).cuda()
+    y_gpu = pk.decompress(buf).cpu().numpy()
+    assert np.array_equal(_bits(y_gpu), _bits(y_cpu)), f"decoded values differ ({bound})"
+    assert violations(x, y_gpu, bound, eps).size == 0
+    return s_cpu
+
+
+SIZES = [1, 31, 32, 33, 4095, 4096, 4097, 3 * 4096 + 17, 20000]
+
+
+@pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_small_fields_all_sizes(pk, orc, bound, dt):
+    for n in SIZES:
+        spec = synth.FieldSpec("t", (n,), "f32" if dt == np.float32 else "f64", 3, A=0.5, tau=0.01)
+        x = synth.generate(spec).numpy()
+        _check(pk, orc, x, bound, 1e-3)
+
+
+@pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+@pytest.mark.parametrize("eps", [1e-1, 1e-4, 0.37])
+def test_adversarial(pk, orc, bound, dt, eps):
+    x = synth.adversarial_f32() if dt == np.float32 else synth.adversarial_f64()
+    _check(pk, orc, x, bound, eps)
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_random_bits_raw_and_constants(pk, orc, dt):
+    rng = np.random.default_rng(7)
+    n = 5 * (16384 // np.dtype(dt).itemsize) + 3
+    u = rng.integers(0, 2**63, size=n, dtype=np.int64).astype(np.uint64)
+    x = (u.astype(np.uint32) if dt == np.float32 else u).view(dt)
+    for bound in ("abs", "rel", "noa"):
+        _check(pk, orc, x, bound, 1e-3)
+        _check(pk, orc, np.full(n, 2.5, dt), bound, 1e-3)
+        _check(pk, orc, np.zeros(n, dt), bound, 1e-3)
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_magnitude_sign_residuals(pk, orc, dt):
+    spec = synth.FieldSpec("t", (40000,), "f32" if dt == np.float32 else "f64", 5, A=1.0, tau=0.01)
+    x = synth.generate(spec).numpy()
+    for bound in ("abs", "rel", "noa"):
+        _check(pk, orc, x, bound, 1e-3, ms=True)
+
+
+def test_empty(pk, orc):
+    for dt in (np.float32, np.float64):
+        for bound in ("abs", "rel", "noa"):
+            x = np.zeros(0, dt)
+            s = pk.compress(torch.zeros(0, dtype=torch.float32 if dt == np.float32 else torch.float64,
+                                        device="cuda"), bound, 1e-3)
+            assert s.cpu().numpy().tobytes() == orc.compress(x, bound, 1e-3)
+
+
+CONFIGS = [("cesm", "abs", 1e-3), ("hurricane", "rel", 1e-3), ("miranda", "abs", 1e-4),
+           ("miranda", "rel", 1e-4), ("miranda", "noa", 1e-4), ("nyx", "abs", 1e-3),
+           ("nyx", "noa", 1e-3)]
+
+
+@pytest.mark.parametrize("name,bound,eps", CONFIGS)
+def test_full_size_configs(pk, orc, name, bound, eps):
+    """BASELINE.json configs at full size, in the launch configuration bench.py
+    times: full stream bytes compared with the oracle (multi-threaded), GPU
+    decode of the oracle stream compared bitwise, exact bound on every element."""
+    spec = synth.CONFIGS[name]
+    xd = synth.generate(spec, device="cuda")
+    x = xd.cpu().numpy()
+    s_gpu = pk.compress(xd, bound, eps).cpu().numpy().tobytes()
+    s_cpu = orc.compress(x, bound, eps, nthreads=max(1, len(__import__("os").sched_getaffinity(0))))
+    assert len(s_gpu) == len(s_cpu) and s_gpu == s_cpu
+    y = pk.decompress(torch.frombuffer(bytearray(s_cpu), dtype=torch.uint8).cuda()).cpu().numpy()
+    y_cpu = orc.decompress(s_cpu, nthreads=8)
+    assert np.array_equal(_bits(y), _bits(y_cpu))
+    assert violations(x, y, bound, eps).size == 0
+
+
+def test_capacity_and_corruption(pk, orc):
+    x = synth.generate(synth.CONFIGS["cesm"], device="cuda", slab=(0, 16))
+    full = pk.compress(x, "abs", 1e-3)
+    out = torch.empty(full.numel() - 1, dtype=torch.uint8, device="cuda")
+    with pytest.raises(pk.PFPLError) as e:
+        pk.compress(x, "abs", 1e-3, out=out)
+    assert e.value.code == -3
+    with pytest.raises(pk.PFPLError):
+        pk.compress(x, "abs", 1e-40)
+    with pytest.raises(pk.PFPLError):
+        pk.decompress(full[:-1].clone())
+    rng = np.random.default_rng(1)
+    for _ in range(100):
+        b = full.clone()
+        i = int(rng.integers(48, b.numel()))
+        b[i] ^= 1 << int(rng.integers(0, 8))
+        try:
+            pk.decompress(b)
+        except pk.PFPLError:
+            pass
+    torch.cuda.synchronize()
+
+
+def test_async_api(pk, orc):
+    x = synth.generate(synth.CONFIGS["cesm"], device="cuda", slab=(0, 32))
+    out = torch.empty(pk.max_compressed_bytes(x.numel(), torch.float32), dtype=torch.uint8,
+                      device="cuda")
+    res = torch.zeros(2, dtype=torch.int64, device="cuda")
+    pk.compress_async(x, out, res, "abs", 1e-3)
+    nb = int(res[0].item())
+    assert out[:nb].cpu().numpy().tobytes() == orc.compress(x.cpu().numpy(), "abs", 1e-3)
+    y = torch.empty_like(x)
+    pk.decompress_async(out[:nb], out[:48].cpu().numpy().tobytes(), y, res)
+    assert int(res[1].item()) == 0
+    assert torch.equal(y, pk.decompress(out[:nb]))
+
+
+@pytest.mark.parametrize("bound", ["abs", "noa"])
+def test_shards_assemble_to_single_stream(pk, orc, bound):
+    """chunk-aligned shards + gathered sizes give a stream
+    byte-identical to the single-device one (P:141 chunks are independent)."""
+    spec = synth.CONFIGS["cesm"]
+    xd = synth.generate(spec, device="cuda")
+    single = pk.compress(xd, bound, 1e-3).cpu().numpy().tobytes()
+    for world in (2, 3):
+        mm = pk.minmax(xd) if bound == "noa" else None
+        parts, tables, hdr = [], [], None
+        for r in range(world):
+            e0, e1 = synth.chunk_slab(spec, r, world)
+            tab, pay, h = pk.compress_shard(xd[e0:e1].contiguous(), e0 // 4096, xd.numel(), bound,
+                                            1e-3, mnmx=mm)
+            tables.append(tab.cpu().numpy().tobytes())
+            parts.append(pay.cpu().numpy().tobytes())
+            hdr = hdr or h
+            assert h == hdr
+        assert hdr + b"".join(tables) + b"".join(parts) == single
