@@ -63,7 +63,7 @@ class Clocks:
 
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+         "clocks_event_reasons.sw_power_cap,utilization.gpu")
 
     def __init__(self, index: int):
         self.index = index
@@ -74,7 +74,7 @@ class Clocks:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                 "--format=csv,noheader,nounits", "-lms", "100"],
+                 "--format=csv,noheader,nounits", "-lms", "50"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -99,9 +99,11 @@ class Clocks:
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:
             f = [x.strip() for x in ln.split(",")]
-            if len(f) < 8:
+            if len(f) < 9:
                 continue
             try:
+                if float(f[8]) < 50:          # keep samples taken under load only
+                    continue
                 sm.append(float(f[1]))
                 mx = float(f[2])
             except ValueError:
@@ -278,6 +280,7 @@ def run_ours(args):
                                                first_chunk, C, out.data_ptr() + 4 * C, pbytes,
                                                y.data_ptr(), nbytes, sh))
 
+    clk = Clocks(local).__enter__()
     # warm-up (also fixes the header / table for the decompress leg)
     for _ in range(max(1, args.warmup)):
         pb = compress_once()
@@ -310,20 +313,28 @@ def run_ours(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    with Clocks(local) as clk:
-        t_wall0 = time.perf_counter()
-        for i in range(args.steps):
-            ev[i][0].record(stream)
-            pb = compress_once()
-            ev[i][1].record(stream)
-            decompress_once(pb)
-            ev[i][2].record(stream)
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-        t_wall = time.perf_counter() - t_wall0
+    t_wall0 = time.perf_counter()
+    for i in range(args.steps):
+        ev[i][0].record(stream)
+        pb = compress_once()
+        ev[i][1].record(stream)
+        decompress_once(pb)
+        ev[i][2].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_wall = time.perf_counter() - t_wall0
     launches = pk.launch_count() - launches0
+    # keep the sampler running while the GPU stays busy with the same work
+    # until it has seen the load (short timed regions end before a 50 ms tick)
+    t_hold = time.perf_counter()
+    while len(clk.lines) < 4 and time.perf_counter() - t_hold < 2.0:
+        for _ in range(10):
+            pb = compress_once()
+            decompress_once(pb)
+        torch.cuda.synchronize()
+    clk.__exit__(None, None, None)
     tc = [ev[i][0].elapsed_time(ev[i][1]) for i in range(args.steps)]
     td = [ev[i][1].elapsed_time(ev[i][2]) for i in range(args.steps)]
     tc_sum, td_sum = sum(tc), sum(td)

@@ -96,17 +96,13 @@ __device__ __forceinline__ void rze1_dec(uint32_t (&lo)[32], uint32_t (&hi)[32],
         if (n & 8u) w |= (uint32_t)z1[r] << 24;
         pw[j] = w;
     }
-    {
-        uint32_t t[KL];
 #pragma unroll
-        for (int j = 0; j < KL; ++j) t[j] = pw[j];
-        transpose_inv<KL>(t, lo);
-    }
+    for (int j = 0; j < KL; ++j) lo[j] = pw[j];
+    transpose_inv<KL>(lo);
     if constexpr (KH > 0) {
-        uint32_t t[KH];
 #pragma unroll
-        for (int j = 0; j < KH; ++j) t[j] = pw[KL + j];
-        transpose_inv<KH>(t, hi);
+        for (int j = 0; j < KH; ++j) hi[j] = pw[KL + j];
+        transpose_inv<KH>(hi);
     } else {
 #pragma unroll
         for (int i = 0; i < 32; ++i) hi[i] = 0;
@@ -209,7 +205,6 @@ __global__ void __launch_bounds__(Tr<T>::NT) decode_kernel(const DecParams p) {
         uint8_t* const dstc = (uint8_t*)p.out + c * (uint64_t)kChunkBytes;
         if (size == rawb) {
             // raw chunk: the stored bytes are the original values
-            copy_raw:
             {
                 const uint8_t* sp = s_buf + delta;
                 for (uint32_t j = tid; j < rawb / 4; j += NT) {

@@ -131,14 +131,19 @@ template <> struct QF<float> {
     // ABS/NOA: a = eps_eff, b = inv, c = eb2.  Bin = rint(v*inv); decode
     // immediately and keep the bin only if |v - bin*2eps| <= eps (R7);
     // |bin| < 2^22 so the zigzag code stays in the denormal range (R8).
+    //
+    // rint without the XU pipe: t = s + 1.5*2^23 rounds s to the nearest integer
+    // (ties to even) for |s| < 2^22 and bits(t) = 0x4B400000 + rint(s); for
+    // |s| >= 2^22 (or inf/NaN) the recovered rb has |rb| >= 2^22 (or is NaN) and
+    // the value is stored losslessly, exactly as with rint.
     __device__ __forceinline__ uint32_t abs_q(float v) const {
         float s = v * b;
-        float rb = rintf(s);
-        bool ok = fabsf(rb) < 4194304.0f;
+        float t = s + 12582912.0f;
+        float rb = t - 12582912.0f;
         float vr = rb * c;
         float diff = fabsf(v - vr);
-        ok = ok && (diff <= a);
-        int32_t bi = __float2int_rz(rb);
+        bool ok = (fabsf(rb) < 4194304.0f) && (diff <= a);
+        int32_t bi = (int32_t)(f2u(t) - 0x4B400000u);
         return ok ? zz(bi) : f2u(v);
     }
     __device__ __forceinline__ float abs_dq(uint32_t w) const {
@@ -183,12 +188,12 @@ template <> struct QF<double> {
     __device__ __forceinline__ void load(const QConst& q) { a = u2d(q.a); b = u2d(q.b); c = u2d(q.c); }
     __device__ __forceinline__ uint64_t abs_q(double v) const {
         double s = v * b;
-        double rb = rint(s);
-        bool ok = fabs(rb) < 2251799813685248.0;
+        double t = s + 6755399441055744.0;          // 1.5 * 2^52
+        double rb = t - 6755399441055744.0;
         double vr = rb * c;
         double diff = fabs(v - vr);
-        ok = ok && (diff <= a);
-        int64_t bi = (int64_t)__double2ll_rz(rb);
+        bool ok = (fabs(rb) < 2251799813685248.0) && (diff <= a);
+        int64_t bi = (int64_t)(d2u(t) - 0x4338000000000000ull);
         return ok ? zz(bi) : d2u(v);
     }
     __device__ __forceinline__ double abs_dq(uint64_t w) const {
@@ -282,15 +287,16 @@ template <int I> __device__ __forceinline__ void xchg(uint32_t& a, uint32_t& b) 
         uint32_t na = __byte_perm(a, b, 0x6240), nb = __byte_perm(a, b, 0x7351);
         a = na; b = nb;
     } else {
+        // mask form: 2 LOP3 + 1 SHF on the ALU pipe, 1 IMAD.SHL on the FMA pipe
         constexpr uint32_t M = I == 0 ? 0x55555555u : I == 1 ? 0x33333333u : 0x0F0F0F0Fu;
         constexpr int s = 1 << I;
-        uint32_t t = ((a >> s) ^ b) & M;
-        b ^= t;
-        a ^= t << s;
+        const uint32_t na = (a & M) | ((b * (1u << s)) & ~M);
+        const uint32_t nb = ((a >> s) & M) | (b & ~M);
+        a = na; b = nb;
     }
 }
 
-template <int K> __device__ __forceinline__ void xchg_all(uint32_t (&o)[K]) {
+template <int K> __device__ __forceinline__ void xchg_all(uint32_t* o) {
 #pragma unroll
     for (int i = 0; (1 << i) < K; ++i) {
 #pragma unroll
@@ -308,26 +314,28 @@ template <int K> __device__ __forceinline__ void xchg_all(uint32_t (&o)[K]) {
     }
 }
 
-template <int K> __device__ __forceinline__ void transpose_fwd(const uint32_t (&in)[32], uint32_t (&o)[K]) {
+// in place: r[0..K-1] receive the K plane words (bit b of the 32 values)
+template <int K> __device__ __forceinline__ void transpose_fwd(uint32_t (&r)[32]) {
     constexpr int H = 32 / K;
 #pragma unroll
     for (int w = 0; w < K; ++w) {
-        uint32_t x = in[w];
+        uint32_t x = r[w];
 #pragma unroll
-        for (int h = 1; h < H; ++h) x |= in[w + K * h] << (K * h);
-        o[w] = x;
+        for (int h = 1; h < H; ++h) x += r[w + K * h] * (1u << (K * h));   // disjoint fields
+        r[w] = x;
     }
-    xchg_all<K>(o);
+    xchg_all<K>(r);
 }
 
-template <int K> __device__ __forceinline__ void transpose_inv(uint32_t (&o)[K], uint32_t (&out)[32]) {
+// in place inverse: r[0..K-1] hold plane words; on return r[0..31] hold values < 2^K
+template <int K> __device__ __forceinline__ void transpose_inv(uint32_t (&r)[32]) {
     constexpr int H = 32 / K;
-    xchg_all<K>(o);
+    xchg_all<K>(r);
 #pragma unroll
     for (int w = 0; w < K; ++w) {
 #pragma unroll
-        for (int h = 0; h < H; ++h)
-            out[w + K * h] = K == 32 ? o[w] : ((o[w] >> (K * h)) & ((1u << (K & 31)) - 1u));
+        for (int h = H - 1; h >= 0; --h)
+            r[w + K * h] = K == 32 ? r[w] : ((r[w] >> (K * h)) & ((1u << (K & 31)) - 1u));
     }
 }
 
@@ -385,6 +393,50 @@ __device__ __forceinline__ uint4 ldg_nc_v4(const void* p) {
     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
     return v;
+}
+
+// ------------------------------------------------------------------------
+// sm_90+/sm_100 asynchronous primitives: mbarrier, TMA, named barriers
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint32_t a, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint32_t a, uint32_t tx) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(tx) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t a) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "LAB_WAIT:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@P1 bra DONE;\n\t"
+        "bra LAB_WAIT;\n"
+        "DONE:\n\t}" ::"r"(a), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void fence_barrier_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// 2-D tiled TMA load into shared memory, completion counted on an mbarrier
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const void* tmap, int x, int y, uint32_t mbar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3}], [%4];" ::"r"(dst), "l"(tmap), "r"(x), "r"(y), "r"(mbar) : "memory");
+}
+__device__ __forceinline__ void prefetch_tmap(const void* tmap) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(tmap) : "memory");
+}
+__device__ __forceinline__ void named_sync(int id, int n) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void named_arrive(int id, int n) {
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
 }  // namespace pfpl

@@ -1,55 +1,53 @@
 // pfpl_encode.cu -- fused PFPL chunk encoder for sm_100a.
 //
-// One CTA per 16 KiB chunk at a time, persistent CTAs that take chunks
-// from an atomic ticket ("dynamically assign the chunks"), all stages
-// fused so the input is read once and the output written once:
-//   load 16 KiB (16-byte coalesced, padded smem rows) -> quantize + verify
-//    -> delta + negabinary -> bit-plane transpose in
-//   registers -> zero-byte elimination with packed warp scans
-//    -> 3 levels of repeated-byte elimination -> raw
-//   fallback -> decoupled look-back for the byte offset ->
-//   realigned 16-byte stores of the payload.
-// Thread t owns elements 32t..32t+31, so its 32 bits of every bit plane form
-// one aligned 32-bit word of the shuffled chunk.
+// Persistent, warp-specialised CTAs.  One 16 KiB chunk is the unit of work
+// (P:141); chunks are taken in order from an atomic ticket (P:158
+// "dynamically assign the chunks").  Every stage is fused so the input is read
+// once and the output written once.
+//
+//   IO warp (1 per CTA)          compute warps (4 for f32, 2 for f64)
+//   -------------------          ------------------------------------
+//   ticket -> TMA 2-D swizzled   wait full[s]; quantize + verify,
+//   load of chunk c into stage   delta + negabinary, bit-plane
+//   s (3-stage ring), arm        transpose in registers,
+//   full[s]                      zero-byte elimination with packed warp scans
+//                                (P:129), 3 repeat levels,
+//   wait ready[s]; decoupled     raw decision; publish the chunk's
+//   look-back; write     aggregate; arrive ready[s]
+//   size table + payload with
+//   16-byte stores; refill s
+//
+// Thread t of the compute warps owns elements 32t..32t+31, so its 32 bits of
+// each bit plane are one aligned word of the shuffled chunk.
+// The payload is assembled in place in the stage buffer: Z1 ends at byte
+// 16384, Z2 | Z3 | Z4 | M4 precede it (section order M4 Z4 Z3 Z2 Z1, R16).
+#include <cuda.h>
 #include "pfpl_device.cuh"
 
 namespace pfpl {
 
-constexpr int ZOFF = 2352;   // Z1 starts here in the assembly buffer; M4|Z4|Z3|Z2 precede it
+constexpr int NSTAGE = 3;
+constexpr int BUFB = 17408;          // 16 KiB + slack; multiple of 1024 (TMA SWIZZLE_128B)
+constexpr int DATAB = 16384;
 
-template <typename T> struct EncGeom {
-    static constexpr int NT = Tr<T>::NT, S = Tr<T>::S;
-    static constexpr int ROWB = 32 * S + 16;                       // padded 32-element row
-    static constexpr int STAGE_IN = NT * ROWB;
-    static constexpr int STAGE = (STAGE_IN > ZOFF + 16384 ? STAGE_IN : ZOFF + 16384) + 32;
+struct StageMeta {
+    unsigned long long c;
+    uint32_t stored, start, raw, pad;
 };
 
-// copy len bytes from shared memory (any alignment) to global memory (any
-// alignment) with 16-byte aligned vector stores for the body (P:166
-// "coalesced memory accesses ... even when writing unaligned compressed data")
-__device__ __forceinline__ void copy_smem_to_global(uint8_t* dst, const uint8_t* src, uint32_t len,
-                                                    int tid, int nt) {
-    const uint32_t mis = (uint32_t)((uintptr_t)dst & 15u);
-    uint32_t head = (16u - mis) & 15u;
-    if (head > len) head = len;
-    const uint32_t body = (len - head) >> 4;
-    const uint32_t tail0 = head + (body << 4);
-    if ((uint32_t)tid < head) dst[tid] = src[tid];
-    if ((uint32_t)tid < len - tail0) dst[tail0 + tid] = src[tail0 + tid];
-    for (uint32_t j = tid; j < body; j += nt) {
-        const uint8_t* s = src + head + (j << 4);
-        const uint32_t a = (uint32_t)__cvta_generic_to_shared(s) & 3u;
-        const uint32_t* sw = (const uint32_t*)(s - a);
-        uint32_t w0 = sw[0], w1 = sw[1], w2 = sw[2], w3 = sw[3], w4 = sw[4];
-        const uint32_t sh = a * 8u;
-        uint4 v;
-        v.x = __funnelshift_r(w0, w1, sh);
-        v.y = __funnelshift_r(w1, w2, sh);
-        v.z = __funnelshift_r(w2, w3, sh);
-        v.w = __funnelshift_r(w3, w4, sh);
-        *(uint4*)(dst + head + (j << 4)) = v;
-    }
-}
+struct EncShared {
+    uint8_t m1[2048];
+    uint8_t m2[256];
+    uint8_t wcnt[4][64];
+    uint16_t off[4][64];
+    unsigned long long wor[4];
+    uint32_t scan[4];
+    uint32_t n1, pad;
+    StageMeta meta[NSTAGE];
+    unsigned long long full[NSTAGE];
+    unsigned long long ready[NSTAGE];
+};
+constexpr int ENC_SMEM = NSTAGE * BUFB + (int)sizeof(EncShared);
 
 __device__ __forceinline__ void put_u64(uint8_t* p, uint64_t v) {
 #pragma unroll
@@ -66,100 +64,6 @@ __device__ void write_header(uint8_t* out, const EncParams& p, const QConst& qc)
     put_u64(out + 40, (uint64_t)kChunkBytes);
 }
 
-// ---------------------------------------------------------------------------
-// level-1 zero-byte elimination over the active bit planes.
-// KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
-// Plane j of the thread holds bit b_j of its 32 residuals; shuffled position
-// of that word: plane p = B-1-b_j, byte offset p*CW/8 + 4*tid (reading R13).
-// ---------------------------------------------------------------------------
-template <typename T, int KL, int KH>
-__device__ __forceinline__ void rze1(const uint32_t (&lo)[32], const uint32_t (&hi)[32],
-                                     uint8_t* s_z1, uint8_t* s_m1, uint8_t (*s_wcnt)[64],
-                                     uint16_t (*s_off)[64], uint32_t* s_n1, int tid, int lane,
-                                     int warp) {
-    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NW = Tr<T>::NW;
-    constexpr int NP = KL + KH;
-    constexpr int NG = NP / 4;
-    uint32_t pw[NP];
-    {
-        uint32_t t[KL];
-        transpose_fwd<KL>(lo, t);
-#pragma unroll
-        for (int j = 0; j < KL; ++j) pw[j] = t[j];
-    }
-    if constexpr (KH > 0) {
-        uint32_t t[KH];
-        transpose_fwd<KH>(hi, t);
-#pragma unroll
-        for (int j = 0; j < KH; ++j) pw[KL + j] = t[j];
-    }
-    uint32_t h[NP];
-#pragma unroll
-    for (int j = 0; j < NP; ++j) h[j] = nzbytes(pw[j]);
-    // per-plane counts (0..4) packed 4 planes per word, 8 bits each (warp totals <= 128)
-    uint32_t ex[NG];
-#pragma unroll
-    for (int g = 0; g < NG; ++g) {
-        uint32_t v = 0;
-#pragma unroll
-        for (int i = 0; i < 4; ++i) v |= ((h[4 * g + i] * 0x01010101u) >> 24) << (8 * i);
-        uint32_t inc = warp_incl_scan(v, lane);
-        ex[g] = inc - v;
-        const int b0 = 4 * g < KL ? 4 * g : 32 + 4 * g - KL;
-        if (lane == 31) *(uint32_t*)&s_wcnt[warp][b0] = inc;
-    }
-    __syncthreads();
-    if (warp == 0) {
-        // plane order = decreasing bit index; lane l owns bit l (and 32+l)
-        uint32_t wl[NW], wh[NW], tl = 0, th = 0;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            wl[w] = lane < KL ? s_wcnt[w][lane] : 0u;
-            wh[w] = lane < KH ? s_wcnt[w][32 + lane] : 0u;
-            tl += wl[w];
-            th += wh[w];
-        }
-        uint32_t sl = tl, sh = th;   // inclusive suffix sums over lanes
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            uint32_t a = __shfl_down_sync(PFPL_FULL, sl, d);
-            uint32_t b = __shfl_down_sync(PFPL_FULL, sh, d);
-            if (lane + d < 32) { sl += a; sh += b; }
-        }
-        const uint32_t tot_h = __shfl_sync(PFPL_FULL, sh, 0);
-        const uint32_t tot_l = __shfl_sync(PFPL_FULL, sl, 0);
-        uint32_t run = tot_h + sl - tl;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            if (lane < KL) s_off[w][lane] = (uint16_t)run;
-            run += wl[w];
-        }
-        run = sh - th;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            if (lane < KH) s_off[w][32 + lane] = (uint16_t)run;
-            run += wh[w];
-        }
-        if (lane == 0) *s_n1 = tot_l + tot_h;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < NP; ++j) {
-        const int b = j < KL ? j : 32 + j - KL;
-        const int pl = B - 1 - b;
-        const uint32_t hj = h[j], w = pw[j];
-        const uint32_t o = s_off[warp][b] + ((ex[j / 4] >> (8 * (j % 4))) & 0xFFu);
-        const uint32_t incl = hj * 0x01010101u;
-        if (hj & 0x1u) s_z1[o] = (uint8_t)w;
-        if (hj & 0x100u) s_z1[o + (incl & 0xFFu)] = (uint8_t)(w >> 8);
-        if (hj & 0x10000u) s_z1[o + ((incl >> 8) & 0xFFu)] = (uint8_t)(w >> 16);
-        if (hj & 0x1000000u) s_z1[o + ((incl >> 16) & 0xFFu)] = (uint8_t)(w >> 24);
-        const uint32_t nb = nib(hj);
-        const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
-        if (!(lane & 1)) s_m1[pl * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
-    }
-}
-
 // scatter the bytes of w whose marker (0x01 per byte in hh) is set to z[o...]
 __device__ __forceinline__ uint32_t scatter_word(uint8_t* z, uint32_t o, uint32_t w, uint32_t hh) {
     const uint32_t incl = hh * 0x01010101u;
@@ -170,184 +74,144 @@ __device__ __forceinline__ uint32_t scatter_word(uint8_t* z, uint32_t o, uint32_
     return o + (incl >> 24);
 }
 
-template <typename T, int MODE, bool MSR>
-__global__ void __launch_bounds__(Tr<T>::NT) encode_kernel(const EncParams p) {
-    typedef typename Tr<T>::W W;
-    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NT = Tr<T>::NT, NW = Tr<T>::NW, S = Tr<T>::S;
-    constexpr int ROWB = EncGeom<T>::ROWB;
-    constexpr int NB2 = 2048 / NT;     // level-2 bytes per thread (16 or 32)
-    constexpr int NWD2 = NB2 / 4;
-
-    __shared__ __align__(16) uint8_t s_stage[EncGeom<T>::STAGE];
-    __shared__ __align__(16) uint8_t s_m1[2048];
-    __shared__ __align__(16) uint8_t s_m2[256];
-    __shared__ __align__(16) uint8_t s_wcnt[NW][64];
-    __shared__ __align__(16) uint16_t s_off[NW][64];
-    __shared__ uint32_t s_scan[NW];
-    __shared__ W s_wor[NW];
-    __shared__ unsigned long long s_c;
-    __shared__ uint32_t s_n1, s_n2, s_start, s_stored, s_write;
-    __shared__ unsigned long long s_dst;
-
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    QConst qc = p.qc;
-    if (MODE == MODE_NOA) qc = *p.qc_dev;
-    QF<T> q;
-    q.load(qc);
-    const bool raw = (qc.flags & HF_RAWWORDS) != 0;
-    uint8_t* const s_z1 = s_stage + ZOFF;
-
-    for (;;) {
-        if (tid == 0) s_c = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-        __syncthreads();
-        const uint64_t c = s_c;
-        if (c >= p.C) break;
-        const uint32_t m = (uint32_t)min((uint64_t)CW, p.n - c * (uint64_t)CW);
-        if (c == 0 && p.write_header && tid == 0) write_header(p.out, p, qc);
-
-        // ---- zero M1, load the chunk into padded rows ----
-        for (int i = tid; i < 2048 / 16; i += NT) ((uint4*)s_m1)[i] = make_uint4(0, 0, 0, 0);
-        const uint8_t* src = (const uint8_t*)p.in + c * (uint64_t)kChunkBytes;
-        if (m == CW) {
+// ---------------------------------------------------------------------------
+// bit shuffle + level-1 zero-byte elimination for one chunk.
+// KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
+// Plane word j holds bit b_j of the thread's 32 residuals; its shuffled
+// position is plane p = B-1-b_j, byte p*CW/8 + 4*tid (reading R13).
+// Z1 (plane-major, non-zero bytes in order) is written to buf[16384-n1, 16384).
+// ---------------------------------------------------------------------------
+template <typename T, int KL, int KH>
+__device__ __forceinline__ void rze1(uint32_t (&lo)[32], uint32_t (&hi)[32], uint8_t* buf,
+                                     EncShared& S, int tid, int lane, int warp) {
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NW = Tr<T>::NW, NTC = Tr<T>::NT;
+    constexpr int NP = KL + KH, NG = NP / 4;
+    transpose_fwd<KL>(lo);
+    if constexpr (KH > 0) transpose_fwd<KH>(hi);
+    auto PW = [&](int j) -> uint32_t { return j < KL ? lo[j] : hi[j - KL]; };
+    // per-plane non-zero byte counts (0..4), 4 planes per word, 8 bits each
+    uint32_t ex[NG];
 #pragma unroll
-            for (int i = 0; i < 1024 / NT; ++i) {
-                const int k = i * NT + tid;
-                const uint4 v = ldg_nc_v4(src + 16 * k);
-                *(uint4*)(s_stage + (k / (2 * S)) * ROWB + (k % (2 * S)) * 16) = v;
-            }
-        } else {
-            // R12: pad a short chunk with its last value -> identical words -> zero residuals
-            for (int e = tid; e < CW; e += NT) {
-                const int se = e < (int)m ? e : (int)m - 1;
-                *(T*)(s_stage + (e / 32) * ROWB + (e % 32) * S) = ((const T*)src)[se];
-            }
+    for (int g = 0; g < NG; ++g) {
+        uint32_t v = 0;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) v += ((nzbytes(PW(4 * g + i)) * 0x01010101u) >> 24) << (8 * i);
+        uint32_t inc = v;
+        if (__any_sync(PFPL_FULL, v != 0)) inc = warp_incl_scan(v, lane);
+        ex[g] = inc - v;
+        const int b0 = 4 * g < KL ? 4 * g : 32 + 4 * g - KL;
+        if (lane == 31) *(uint32_t*)&S.wcnt[warp][b0] = inc;
+    }
+    named_sync(1, NTC);
+    if (warp == 0) {
+        // plane order = decreasing bit index; lane l owns bit l (and 32+l)
+        uint32_t wl[NW], wh[NW], tl = 0, th = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) {
+            wl[w] = lane < KL ? S.wcnt[w][lane] : 0u;
+            wh[w] = lane < KH ? S.wcnt[w][32 + lane] : 0u;
+            tl += wl[w];
+            th += wh[w];
         }
-        __syncthreads();
-
-        // ---- quantize + verify ----
-        W qv[32];
-        {
-            const uint4* row = (const uint4*)(s_stage + tid * ROWB);
+        uint32_t sl = tl, sh = th;   // inclusive suffix sums over lanes
 #pragma unroll
-            for (int j = 0; j < 2 * S; ++j) {
-                const uint4 v = row[j];
-                T x[16 / S];
-                memcpy(x, &v, 16);
-#pragma unroll
-                for (int i = 0; i < 16 / S; ++i) qv[j * (16 / S) + i] = quantize<T, MODE>(q, x[i], raw);
-            }
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t a = __shfl_down_sync(PFPL_FULL, sl, d);
+            const uint32_t b = KH > 0 ? __shfl_down_sync(PFPL_FULL, sh, d) : 0u;
+            if (lane + d < 32) { sl += a; sh += b; }
         }
-        // ---- delta (predecessor of the first value is 0) + residual code ----
-        W qprev = __shfl_up_sync(PFPL_FULL, qv[31], 1);
-        if (lane == 0) {
-            qprev = 0;
-            if (tid > 0) qprev = quantize<T, MODE>(q, *(const T*)(s_stage + (tid - 1) * ROWB + 31 * S), raw);
-        }
-        uint32_t lo[32], hi[32];
-        W orv = 0;
+        const uint32_t tot_h = KH > 0 ? __shfl_sync(PFPL_FULL, sh, 0) : 0u;
+        const uint32_t tot_l = __shfl_sync(PFPL_FULL, sl, 0);
+        uint32_t run = tot_h + sl - tl;
 #pragma unroll
-        for (int i = 0; i < 32; ++i) {
-            const W r = rcode<MSR>((W)(qv[i] - (i ? qv[i - 1] : qprev)));
-            orv |= r;
-            lo[i] = (uint32_t)r;
-            hi[i] = sizeof(W) == 8 ? (uint32_t)((uint64_t)r >> 32) : 0u;
+        for (int w = 0; w < NW; ++w) {
+            if (lane < KL) S.off[w][lane] = (uint16_t)run;
+            run += wl[w];
         }
-        {
-            const uint32_t ol = __reduce_or_sync(PFPL_FULL, (uint32_t)orv);
-            const uint32_t oh = sizeof(W) == 8 ? __reduce_or_sync(PFPL_FULL, (uint32_t)((uint64_t)orv >> 32)) : 0u;
-            if (lane == 0) s_wor[warp] = (W)((sizeof(W) == 8 ? ((uint64_t)oh << 32) : 0ull) | ol);
-        }
-        __syncthreads();   // all rows consumed; active planes known
-        uint64_t bor = 0;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) bor |= (uint64_t)s_wor[w];
-        const int P = bor ? 64 - __clzll((long long)bor) : 0;   // number of active low bits
-
-        // ---- bit shuffle + level-1 zero elimination (block-uniform tier) ----
-        if (P == 0) {
-            if (tid == 0) s_n1 = 0;
-        } else if (B == 32 || P <= 32) {
-            if (P <= 4) rze1<T, 4, 0>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 8) rze1<T, 8, 0>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 16) rze1<T, 16, 0>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else rze1<T, 32, 0>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-        } else {
-            if (P <= 36) rze1<T, 32, 4>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 40) rze1<T, 32, 8>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 48) rze1<T, 32, 16>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else rze1<T, 32, 32>(lo, hi, s_z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-        }
-        __syncthreads();
-
-        // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 256 B + Z2) ----
-        {
-            uint32_t w2[NWD2], h2[NWD2];
-            const uint32_t* m1w = (const uint32_t*)s_m1;
-#pragma unroll
-            for (int i = 0; i < NWD2; i += 4) {
-                const uint4 v = *(const uint4*)(m1w + NWD2 * tid + i);
-                w2[i] = v.x; w2[i + 1] = v.y; w2[i + 2] = v.z; w2[i + 3] = v.w;
-            }
-            const uint32_t pred = tid ? m1w[NWD2 * tid - 1] : 0u;
-            uint32_t bits2 = 0;
-#pragma unroll
-            for (int i = 0; i < NWD2; ++i) {
-                const uint32_t pw = i ? w2[i - 1] : pred;
-                h2[i] = nzbytes(w2[i] ^ __funnelshift_l(pw, w2[i], 8));
-                bits2 |= nib(h2[i]) << (4 * i);
-            }
-            const uint32_t cnt2 = __popc(bits2);
-            const uint32_t inc = warp_incl_scan(cnt2, lane);
-            if (lane == 31) s_scan[warp] = inc;
-            __syncthreads();
-            uint32_t base = 0, n2 = 0;
+        if (KH > 0) {
+            run = sh - th;
 #pragma unroll
             for (int w = 0; w < NW; ++w) {
-                const uint32_t v = s_scan[w];
-                if (w < warp) base += v;
-                n2 += v;
+                if (lane < KH) S.off[w][32 + lane] = (uint16_t)run;
+                run += wh[w];
             }
-            if (cnt2) {
-                uint8_t* z2 = s_z1 - n2;
-                uint32_t o = base + inc - cnt2;
-#pragma unroll
-                for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
-            }
-            if (NB2 == 16) ((uint16_t*)s_m2)[tid] = (uint16_t)bits2;
-            else ((uint32_t*)s_m2)[tid] = bits2;
-            if (tid == 0) s_n2 = n2;
         }
-        __syncthreads();
+        if (lane == 0) S.n1 = tot_l + tot_h;
+    }
+    named_sync(1, NTC);
+    uint8_t* z1 = buf + DATAB - S.n1;
+#pragma unroll
+    for (int j = 0; j < NP; ++j) {
+        const uint32_t w = PW(j);
+        if (!__any_sync(PFPL_FULL, w != 0)) continue;          // warp-uniform skip of empty planes
+        const int b = j < KL ? j : 32 + j - KL;
+        const int pl = B - 1 - b;
+        const uint32_t hj = nzbytes(w);
+        const uint32_t o = S.off[warp][b] + ((ex[j / 4] >> (8 * (j % 4))) & 0xFFu);
+        scatter_word(z1, o, w, hj);
+        const uint32_t nb = nib(hj);
+        const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
+        if (!(lane & 1)) S.m1[pl * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
+    }
+}
 
-        // ---- levels 3 and 4, size, raw decision, look-back (warp 0) ----
-        if (warp == 0) {
-            const uint32_t n1 = s_n1, n2 = s_n2;
-            const uint2 v = ((const uint2*)s_m2)[lane];
-            const uint32_t pred = lane ? ((const uint32_t*)s_m2)[2 * lane - 1] : 0u;
-            const uint32_t h0 = nzbytes(v.x ^ __funnelshift_l(pred, v.x, 8));
-            const uint32_t h1 = nzbytes(v.y ^ __funnelshift_l(v.x, v.y, 8));
-            const uint32_t m3 = nib(h0) | (nib(h1) << 4);
-            const uint32_t cnt3 = __popc(m3);
-            const uint32_t inc3 = warp_incl_scan(cnt3, lane);
-            const uint32_t n3 = __shfl_sync(PFPL_FULL, inc3, 31);
-            uint8_t* z3 = s_z1 - n2 - n3;
-            scatter_word(z3, scatter_word(z3, inc3 - cnt3, v.x, h0), v.y, h1);
-            // level 4 on M3 (32 bytes, one per lane)
-            uint32_t pm3 = __shfl_up_sync(PFPL_FULL, m3, 1);
-            if (lane == 0) pm3 = 0;
-            const bool dif = m3 != pm3;
-            const uint32_t M4 = __ballot_sync(PFPL_FULL, dif);
-            const uint32_t n4 = __popc(M4);
-            uint8_t* z4 = s_z1 - n2 - n3 - n4;
-            if (dif) z4[__popc(M4 & ((1u << lane) - 1u))] = (uint8_t)m3;
-            if (lane < 4) z4[lane - 4] = (uint8_t)(M4 >> (8 * lane));
-            const uint32_t size = 4 + n4 + n3 + n2 + n1;
-            const uint32_t rawb = m * S;
-            const bool israw = size >= rawb;             // P:158
-            const uint32_t stored = israw ? rawb : size;
-            // decoupled look-back
-            const uint64_t EP = (uint64_t)p.epoch << 48;
-            if (lane == 0) st_relaxed(&p.status[c], EP | ((c == 0 ? LB_P : LB_A) << 46) | stored);
+template <typename T, int MODE, bool MSR>
+__global__ void __launch_bounds__(Tr<T>::NT + 32, 4)
+encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
+    typedef typename Tr<T>::W W;
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;
+    constexpr int NB2 = 2048 / NTC;     // level-2 bytes per compute thread (16 or 32)
+    constexpr int NWD2 = NB2 / 4;
+
+    extern __shared__ __align__(1024) uint8_t smem[];
+    EncShared& S = *reinterpret_cast<EncShared*>(smem + NSTAGE * BUFB);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+
+    QConst qc = p.qc;
+    if (MODE == MODE_NOA) qc = *p.qc_dev;
+
+    if (tid == 0) {
+        if (smem_u32(smem) & 1023u) __trap();       // TMA SWIZZLE_128B needs 1024-byte alignment
+        for (int s = 0; s < NSTAGE; ++s) {
+            mbar_init(smem_u32(&S.full[s]), 1);
+            mbar_init(smem_u32(&S.ready[s]), 1);
+        }
+        fence_barrier_init();
+    }
+    __syncthreads();
+
+    if (warp == NWC) {
+        // =========================== IO warp ===========================
+        const uint64_t C = p.C;
+        const uint64_t full_chunks = p.n / CW;
+        unsigned long long next = 0;
+        auto issue = [&](int s, unsigned long long t) {
+            S.meta[s].c = t;
+            if (t < full_chunks) {
+                fence_proxy_async();
+                mbar_arrive_tx(smem_u32(&S.full[s]), DATAB);
+                tma_load_2d(smem_u32(smem + s * BUFB), &tmap, 0, (int)(t * 128), smem_u32(&S.full[s]));
+            } else {
+                mbar_arrive(smem_u32(&S.full[s]));       // tail chunk (compute loads it) or end
+            }
+        };
+        if (lane == 0) {
+            prefetch_tmap(&tmap);
+            for (int s = 0; s < NSTAGE; ++s) issue(s, atomicAdd(p.ticket, 1ull) - p.ticket_base);
+            next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+        }
+        __syncwarp();
+        const uint64_t EP = (uint64_t)p.epoch << 48;
+        for (uint32_t it = 0;; ++it) {
+            const int s = it % NSTAGE;
+            const uint32_t ph = (it / NSTAGE) & 1u;
+            const uint64_t c = S.meta[s].c;
+            if (c >= C) break;
+            mbar_wait(smem_u32(&S.ready[s]), ph);
+            const uint32_t stored = S.meta[s].stored;
+            uint32_t start = S.meta[s].start;
+            const uint32_t israw = S.meta[s].raw;
+            // ---- decoupled look-back; the aggregate was published by compute ----
             uint64_t excl = 0;
             if (c > 0) {
                 int64_t look = (int64_t)c - 1;
@@ -372,30 +236,243 @@ __global__ void __launch_bounds__(Tr<T>::NT) encode_kernel(const EncParams p) {
                 }
                 if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + stored));
             }
+            const uint64_t dst = p.payload_off + excl;
             if (lane == 0) {
-                const uint64_t dst = p.payload_off + excl;
                 p.table[c] = stored;
-                if (c == p.C - 1) p.result[0] = dst + stored;
-                s_dst = dst;
-                s_stored = stored;
-                s_start = israw ? 0u : (uint32_t)(ZOFF - 4 - n4 - n3 - n2);
-                s_write = (dst + stored <= p.cap) ? (israw ? 2u : 1u) : 0u;
+                if (c == C - 1) p.result[0] = dst + stored;
+                if (c == 0 && p.write_header) write_header(p.out, p, qc);
+            }
+            uint8_t* buf = smem + s * BUFB;
+            if (dst + stored <= p.cap) {
+                if (israw) {
+                    // raw chunk (R17): stage the original bytes, aligned
+                    const uint8_t* src = (const uint8_t*)p.in + c * (uint64_t)kChunkBytes;
+                    for (uint32_t i = lane; i < stored / 16; i += 32) ((uint4*)buf)[i] = ldg_nc_v4(src + 16 * i);
+                    for (uint32_t i = (stored / 16) * 4 + lane; i < stored / 4; i += 32)
+                        ((uint32_t*)buf)[i] = ((const uint32_t*)src)[i];
+                    __syncwarp();
+                    start = 0;
+                }
+                // 16-byte aligned stores for the body (coalesced even for
+                // unaligned compressed data), bytes for the head and tail
+                uint8_t* o = p.out + dst;
+                const uint8_t* src = buf + start;
+                const uint32_t mis = (uint32_t)((uintptr_t)o & 15u);
+                uint32_t head = (16u - mis) & 15u;
+                if (head > stored) head = stored;
+                const uint32_t body = (stored - head) >> 4;
+                const uint32_t tail0 = head + (body << 4);
+                if ((uint32_t)lane < head) o[lane] = src[lane];
+                if ((uint32_t)lane < stored - tail0) o[tail0 + lane] = src[tail0 + lane];
+                for (uint32_t j = lane; j < body; j += 32) {
+                    const uint8_t* sp = src + head + (j << 4);
+                    const uint32_t a = smem_u32(sp) & 3u;
+                    const uint32_t* sw = (const uint32_t*)(sp - a);
+                    const uint32_t w0 = sw[0], w1 = sw[1], w2 = sw[2], w3 = sw[3], w4 = sw[4];
+                    const uint32_t sh = a * 8u;
+                    uint4 v;
+                    v.x = __funnelshift_r(w0, w1, sh);
+                    v.y = __funnelshift_r(w1, w2, sh);
+                    v.z = __funnelshift_r(w2, w3, sh);
+                    v.w = __funnelshift_r(w3, w4, sh);
+                    *(uint4*)(o + head + (j << 4)) = v;
+                }
+            }
+            __syncwarp();
+            if (lane == 0) {
+                const unsigned long long t = next;
+                next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+                issue(s, t);
+            }
+            __syncwarp();
+        }
+        return;
+    }
+
+    // ============================ compute warps ============================
+    QF<T> q;
+    q.load(qc);
+    const bool raw = (qc.flags & HF_RAWWORDS) != 0;
+    for (uint32_t it = 0;; ++it) {
+        const int s = it % NSTAGE;
+        const uint32_t ph = (it / NSTAGE) & 1u;
+        mbar_wait(smem_u32(&S.full[s]), ph);
+        const uint64_t c = S.meta[s].c;
+        if (c >= p.C) break;
+        uint8_t* buf = smem + s * BUFB;
+        const uint32_t m = (uint32_t)min((uint64_t)CW, p.n - c * (uint64_t)CW);
+
+        // zero this thread's part of M1
+#pragma unroll
+        for (int i = 0; i < 2048 / 16 / NTC; ++i)
+            ((uint4*)S.m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
+
+        // ---- quantize + verify, delta, residual code ----
+        uint32_t lo[32], hi[32];
+        W orv = 0;
+        {
+            W qprev = 0;
+            if (m == CW) {
+                if (tid > 0) {
+                    T pv;
+                    if (sizeof(T) == 4) {
+                        const int r = tid - 1;
+                        pv = *(const T*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 12);
+                    } else {
+                        const int r = 2 * tid - 1;
+                        pv = *(const T*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 8);
+                    }
+                    qprev = quantize<T, MODE>(q, pv, raw);
+                }
+#pragma unroll
+                for (int i = 0; i < 2 * S_; ++i) {
+                    const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                    const uint4 v = *(const uint4*)(buf + r * 128 + (((i & 7) ^ (r & 7)) << 4));
+                    T x[16 / S_];
+                    memcpy(x, &v, 16);
+#pragma unroll
+                    for (int k = 0; k < 16 / S_; ++k) {
+                        const W qw = quantize<T, MODE>(q, x[k], raw);
+                        const W r2 = rcode<MSR>((W)(qw - qprev));
+                        qprev = qw;
+                        orv |= r2;
+                        lo[i * (16 / S_) + k] = (uint32_t)r2;
+                        hi[i * (16 / S_) + k] = sizeof(W) == 8 ? (uint32_t)((uint64_t)r2 >> 32) : 0u;
+                    }
+                }
+            } else {
+                // tail chunk: plain loads; R12 pads with the last value -> zero residuals
+                const T* src = (const T*)p.in + c * (uint64_t)CW;
+                if (tid > 0) qprev = quantize<T, MODE>(q, src[min(32 * tid - 1, (int)m - 1)], raw);
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                    const W qw = quantize<T, MODE>(q, src[min(32 * tid + i, (int)m - 1)], raw);
+                    const W r2 = rcode<MSR>((W)(qw - qprev));
+                    qprev = qw;
+                    orv |= r2;
+                    lo[i] = (uint32_t)r2;
+                    hi[i] = sizeof(W) == 8 ? (uint32_t)((uint64_t)r2 >> 32) : 0u;
+                }
             }
         }
-        __syncthreads();
-        const uint32_t wr = s_write;
-        if (wr == 2) {
-            // raw chunk: original input bytes (R17); stage them aligned
-            const uint32_t nb = m * S;
-            for (uint32_t i = tid; i < nb / 16; i += NT) ((uint4*)s_stage)[i] = ldg_nc_v4(src + 16 * i);
-            for (uint32_t i = (nb / 16) * 4 + tid; i < nb / 4; i += NT)
-                ((uint32_t*)s_stage)[i] = ((const uint32_t*)src)[i];
-            __syncthreads();
+        {
+            const uint32_t ol = __reduce_or_sync(PFPL_FULL, (uint32_t)orv);
+            const uint32_t oh = sizeof(W) == 8 ? __reduce_or_sync(PFPL_FULL, (uint32_t)((uint64_t)orv >> 32)) : 0u;
+            if (lane == 0) S.wor[warp] = ((unsigned long long)oh << 32) | ol;
         }
-        if (wr) copy_smem_to_global(p.out + s_dst, s_stage + s_start, s_stored, tid, NT);
+        named_sync(1, NTC);    // rows consumed, M1 zeroed, active planes known
+        unsigned long long bor = 0;
+#pragma unroll
+        for (int w = 0; w < NWC; ++w) bor |= S.wor[w];
+        const int P = bor ? 64 - __clzll((long long)bor) : 0;
+
+        // ---- bit shuffle + level-1 zero elimination (block-uniform tier) ----
+        if (P == 0) {
+            if (tid == 0) S.n1 = 0;
+        } else if (B == 32 || P <= 32) {
+            if (P <= 4) rze1<T, 4, 0>(lo, hi, buf, S, tid, lane, warp);
+            else if (P <= 8) rze1<T, 8, 0>(lo, hi, buf, S, tid, lane, warp);
+            else if (P <= 16) rze1<T, 16, 0>(lo, hi, buf, S, tid, lane, warp);
+            else rze1<T, 32, 0>(lo, hi, buf, S, tid, lane, warp);
+        } else {
+            if (P <= 36) rze1<T, 32, 4>(lo, hi, buf, S, tid, lane, warp);
+            else if (P <= 40) rze1<T, 32, 8>(lo, hi, buf, S, tid, lane, warp);
+            else if (P <= 48) rze1<T, 32, 16>(lo, hi, buf, S, tid, lane, warp);
+            else rze1<T, 32, 32>(lo, hi, buf, S, tid, lane, warp);
+        }
+        named_sync(1, NTC);    // Z1 and M1 complete
+
+        // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 + Z2) ----
+        const uint32_t n1 = S.n1;
+        uint32_t n2 = 0;
+        {
+            uint32_t w2[NWD2], h2[NWD2];
+            const uint32_t* m1w = (const uint32_t*)S.m1;
+#pragma unroll
+            for (int i = 0; i < NWD2; i += 4) {
+                const uint4 v = *(const uint4*)(m1w + NWD2 * tid + i);
+                w2[i] = v.x; w2[i + 1] = v.y; w2[i + 2] = v.z; w2[i + 3] = v.w;
+            }
+            const uint32_t pred = tid ? m1w[NWD2 * tid - 1] : 0u;
+            uint32_t bits2 = 0;
+#pragma unroll
+            for (int i = 0; i < NWD2; ++i) {
+                const uint32_t pw = i ? w2[i - 1] : pred;
+                h2[i] = nzbytes(w2[i] ^ __funnelshift_l(pw, w2[i], 8));
+                bits2 |= nib(h2[i]) << (4 * i);
+            }
+            const uint32_t cnt2 = __popc(bits2);
+            uint32_t inc = cnt2;
+            if (__any_sync(PFPL_FULL, cnt2 != 0)) inc = warp_incl_scan(cnt2, lane);
+            if (lane == 31) S.scan[warp] = inc;
+            named_sync(1, NTC);
+            uint32_t base = 0;
+#pragma unroll
+            for (int w = 0; w < NWC; ++w) {
+                const uint32_t v = S.scan[w];
+                if (w < warp) base += v;
+                n2 += v;
+            }
+            if (cnt2 && n1 + n2 <= (uint32_t)DATAB) {
+                uint8_t* z2 = buf + DATAB - n1 - n2;
+                uint32_t o = base + inc - cnt2;
+#pragma unroll
+                for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
+            }
+            if (NB2 == 16) ((uint16_t*)S.m2)[tid] = (uint16_t)bits2;
+            else ((uint32_t*)S.m2)[tid] = bits2;
+        }
+        fence_proxy_async();   // generic writes to the stage buffer before its next TMA refill
+        if (warp != 0) {
+            named_arrive(2, NTC);
+            continue;
+        }
+        named_sync(2, NTC);
+
+        // ---- levels 3 and 4, size, raw decision (warp 0) ----
+        {
+            const uint2 v = ((const uint2*)S.m2)[lane];
+            const uint32_t pred = lane ? ((const uint32_t*)S.m2)[2 * lane - 1] : 0u;
+            const uint32_t h0 = nzbytes(v.x ^ __funnelshift_l(pred, v.x, 8));
+            const uint32_t h1 = nzbytes(v.y ^ __funnelshift_l(v.x, v.y, 8));
+            const uint32_t m3 = nib(h0) | (nib(h1) << 4);
+            const uint32_t cnt3 = __popc(m3);
+            const uint32_t inc3 = warp_incl_scan(cnt3, lane);
+            const uint32_t n3 = __shfl_sync(PFPL_FULL, inc3, 31);
+            uint32_t pm3 = __shfl_up_sync(PFPL_FULL, m3, 1);
+            if (lane == 0) pm3 = 0;
+            const bool dif = m3 != pm3;
+            const uint32_t M4 = __ballot_sync(PFPL_FULL, dif);
+            const uint32_t n4 = __popc(M4);
+            const uint32_t size = 4 + n4 + n3 + n2 + n1;
+            const bool fits = size <= (uint32_t)DATAB;
+            if (fits) {
+                uint8_t* z3 = buf + DATAB - n1 - n2 - n3;
+                scatter_word(z3, scatter_word(z3, inc3 - cnt3, v.x, h0), v.y, h1);
+                uint8_t* z4 = z3 - n4;
+                if (dif) z4[__popc(M4 & ((1u << lane) - 1u))] = (uint8_t)m3;
+                if (lane < 4) z4[lane - 4] = (uint8_t)(M4 >> (8 * lane));
+            }
+            const uint32_t rawb = m * S_;
+            const bool israw = size >= rawb;             // P:158
+            const uint32_t stored = israw ? rawb : size;
+            fence_proxy_async();
+            __syncwarp();
+            if (lane == 0) {
+                S.meta[s].stored = stored;
+                S.meta[s].start = fits ? (uint32_t)DATAB - size : 0u;
+                S.meta[s].raw = israw ? 1u : 0u;
+                const uint64_t EP = (uint64_t)p.epoch << 48;
+                st_relaxed(&p.status[c], EP | ((c == 0 ? LB_P : LB_A) << 46) | stored);
+                mbar_arrive(smem_u32(&S.ready[s]));
+            }
+        }
     }
 }
 
+// ---------------------------------------------------------------------------
+// host side
+// ---------------------------------------------------------------------------
 template <typename T, int MODE, bool MSR>
 static void* enc_fn() { return (void*)encode_kernel<T, MODE, MSR>; }
 
@@ -411,6 +488,12 @@ static void* pick_enc(int dtype, int mode, bool ms) {
 #undef PFPL_E
 }
 
+static int enc_threads(int dtype) { return (dtype == 0 ? Tr<float>::NT : Tr<double>::NT) + 32; }
+
+static cudaError_t prepare_enc(void* fn) {
+    return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ENC_SMEM);
+}
+
 int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
     static int cache[2][4][2] = {};
     int& g = cache[dtype][mode][ms];
@@ -418,18 +501,64 @@ int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
         int dev = 0, sms = 148, per = 1;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        const int nt = dtype == 0 ? Tr<float>::NT : Tr<double>::NT;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, pick_enc(dtype, mode, ms), nt, 0);
+        void* fn = pick_enc(dtype, mode, ms);
+        prepare_enc(fn);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, enc_threads(dtype), ENC_SMEM);
         g = sms * (per > 0 ? per : 1);
     }
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
 }
 
+int encode_stages() { return NSTAGE; }
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn get_encode_tiled() {
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        void* f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (EncodeTiledFn)f;
+    }
+    return fn;
+}
+
+// 2-D view of the input as 128-byte rows of 32 u32 words; a chunk = 128 rows.
+cudaError_t make_row_tmap(const void* base, uint64_t bytes, CUtensorMap* map) {
+    memset(map, 0, sizeof(*map));
+    const uint64_t rows = bytes / 128;
+    if (rows < 128) return cudaSuccess;            // no full chunk: map never used
+    EncodeTiledFn fn = get_encode_tiled();
+    if (!fn) return cudaErrorNotSupported;
+    cuuint64_t dims[2] = {32, rows};
+    cuuint64_t strides[1] = {128};
+    cuuint32_t box[2] = {32, 128};
+    cuuint32_t es[2] = {1, 1};
+    CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(base), dims, strides,
+                    box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
 cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int grid,
                           cudaStream_t s) {
-    const int nt = dtype == 0 ? Tr<float>::NT : Tr<double>::NT;
-    void* args[] = {(void*)&p};
-    return cudaLaunchKernel(pick_enc(dtype, mode, ms), dim3(grid), dim3(nt), args, 0, s);
+    alignas(64) CUtensorMap map;
+    cudaError_t e = make_row_tmap(p.in, p.n * (dtype == 0 ? 4u : 8u), &map);
+    if (e != cudaSuccess) return e;
+    void* fn = pick_enc(dtype, mode, ms);
+    static bool prepared[2][4][2] = {};
+    if (!prepared[dtype][mode][ms]) {
+        e = prepare_enc(fn);
+        if (e != cudaSuccess) return e;
+        prepared[dtype][mode][ms] = true;
+    }
+    void* args[] = {(void*)&p, (void*)&map};
+    return cudaLaunchKernel(fn, dim3(grid), dim3(enc_threads(dtype)), args, ENC_SMEM, s);
 }
 
 }  // namespace pfpl

@@ -76,6 +76,7 @@ cudaError_t launch_header_only(uint8_t* out, uint64_t n, int dtype, int bound, d
                                const QConst qc, const QConst* qc_dev, uint64_t* result,
                                cudaStream_t s);
 int encode_grid(int dtype, int mode, bool ms, uint64_t C);
+int encode_stages();
 int decode_grid(int dtype, int mode, bool ms, uint64_t C);
 
 // host-side portable log2 (same operation sequence as the device code)
