@@ -5,34 +5,39 @@
 // "dynamically assign the chunks").  Every stage is fused so the input is read
 // once and the output written once.
 //
-//   IO warp (1 per CTA)          compute warps (4 for f32, 2 for f64)
-//   -------------------          ------------------------------------
-//   ticket -> TMA 2-D swizzled   wait full[s]; quantize + verify,
-//   load of chunk c into stage   delta + negabinary, bit-plane
-//   s (3-stage ring), arm        transpose in registers,
-//   full[s]                      zero-byte elimination with packed warp scans
-//                                (P:129), 3 repeat levels,
-//   wait ready[s]; decoupled     raw decision; publish the chunk's
-//   look-back; write     aggregate; arrive ready[s]
-//   size table + payload with
-//   16-byte stores; refill s
+//   compute warps (4 for f32, 2 for f64)          IO warp (1 per CTA)
+//   ------------------------------------          -------------------
+//   wait full[s]; read rows of chunk c from the   pop (chunk, arena slice) from
+//   TMA-swizzled stage s; warp 0 refills s with   the queue; decoupled look-back
+//   the next ticket's chunk (TMA, 2-stage ring);  for the byte offset;
+//   quantize + verify, delta +         size table entry; copy the
+//   negabinary, bit-plane transpose in    payload (or the raw chunk,
+//   registers, zero-byte           P:158) to HBM with 16-byte
+//   elimination with packed warp scans (P:129,    stores; release the arena
+//   P:164) into a reserved arena slice, 3 repeat  slice
+//   levels, raw decision; publish
+//   the aggregate; push (chunk, slice) to the IO
 //
+// Input refills never wait for output: payloads live in a per-CTA circular
+// arena, so a slow look-back only delays the IO warp.
 // Thread t of the compute warps owns elements 32t..32t+31, so its 32 bits of
-// each bit plane are one aligned word of the shuffled chunk (DESIGN.md 7).
-// The payload is assembled in place in the stage buffer: Z1 ends at byte
-// 16384, Z2 | Z3 | Z4 | M4 precede it (section order M4 Z4 Z3 Z2 Z1, R16).
+// each bit plane are one aligned word of the shuffled chunk (DESIGN.md 7.1).
+// Arena slice of a chunk: [pos, pos + ZPRE + n1) with Z1 at pos + ZPRE and
+// M4 | Z4 | Z3 | Z2 packed immediately before it (section order of R16).
 #include <cuda.h>
 #include "pfpl_device.cuh"
 
 namespace pfpl {
 
-constexpr int NSTAGE = 3;
-constexpr int BUFB = 17408;          // 16 KiB + slack; multiple of 1024 (TMA SWIZZLE_128B)
-constexpr int DATAB = 16384;
+constexpr int NIN = 2;               // input stages (TMA ring)
+constexpr int DATAB = 16384;         // bytes per chunk
+constexpr int ZPRE = 2352;           // >= 4 + 32 + 256 + 2048, multiple of 16
+constexpr int NQ = 8;                // IO queue depth
+constexpr int ARENA = 20800;         // circular payload arena (bytes, multiple of 16)
 
-struct StageMeta {
+struct QEntry {
     unsigned long long c;
-    uint32_t stored, start, raw, pad;
+    uint32_t start, stored, raw, rend;
 };
 
 struct EncShared {
@@ -42,12 +47,16 @@ struct EncShared {
     uint16_t off[4][64];
     unsigned long long wor[4];
     uint32_t scan[4];
-    uint32_t n1, pad;
-    StageMeta meta[NSTAGE];
-    unsigned long long full[NSTAGE];
-    unsigned long long ready[NSTAGE];
+    uint32_t n1, apos, head, tail;
+    unsigned long long in_c[NIN];
+    QEntry q[NQ];
+    unsigned long long full[NIN], mq_full[NQ], mq_empty[NQ];
 };
-constexpr int ENC_SMEM = NSTAGE * BUFB + (int)sizeof(EncShared);
+constexpr int ARENA_OFF = NIN * DATAB;
+constexpr int SHARED_OFF = ARENA_OFF + ARENA + 64;
+constexpr int ENC_SMEM = SHARED_OFF + (int)sizeof(EncShared);
+static_assert(ENC_SMEM <= 57344, "4 CTAs per SM need <= 56 KiB of shared memory each");
+static_assert(ZPRE + DATAB <= ARENA, "the arena must hold a worst-case chunk");
 
 __device__ __forceinline__ void put_u64(uint8_t* p, uint64_t v) {
 #pragma unroll
@@ -79,10 +88,26 @@ __device__ __forceinline__ uint32_t scatter_word(uint8_t* z, uint32_t o, uint32_
 // KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
 // Plane word j holds bit b_j of the thread's 32 residuals; its shuffled
 // position is plane p = B-1-b_j, byte p*CW/8 + 4*tid (reading R13).
-// Z1 (plane-major, non-zero bytes in order) is written to buf[16384-n1, 16384).
+// Z1 (plane-major, non-zero bytes in order) goes to the chunk's arena slice.
 // ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
+    return *(const volatile uint32_t*)p;
+}
+
+// reserve ZPRE + n1 bytes of the arena (compute warp 0, lane 0); waits only if
+// the IO warp lags by more than the arena's capacity
+__device__ __forceinline__ void reserve_arena(EncShared& S, uint32_t n1) {
+    const uint32_t R = (ZPRE + n1 + 15u) & ~15u;
+    uint32_t head = S.head;
+    const uint32_t p0 = head % ARENA;
+    if (p0 + R > (uint32_t)ARENA) head += ARENA - p0;      // do not wrap a slice
+    while (head + R - ld_volatile_u32(&S.tail) > (uint32_t)ARENA) __nanosleep(64);
+    S.apos = head % ARENA;
+    S.head = head + R;
+}
+
 template <typename T, int KL, int KH>
-__device__ __forceinline__ void rze1(uint32_t (&lo)[32], uint32_t (&hi)[32], uint8_t* buf,
+__device__ __forceinline__ void rze1(uint32_t (&lo)[32], uint32_t (&hi)[32], uint8_t* arena,
                                      EncShared& S, int tid, int lane, int warp) {
     constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NW = Tr<T>::NW, NTC = Tr<T>::NT;
     constexpr int NP = KL + KH, NG = NP / 4;
@@ -136,10 +161,13 @@ __device__ __forceinline__ void rze1(uint32_t (&lo)[32], uint32_t (&hi)[32], uin
                 run += wh[w];
             }
         }
-        if (lane == 0) S.n1 = tot_l + tot_h;
+        if (lane == 0) {
+            S.n1 = tot_l + tot_h;
+            reserve_arena(S, tot_l + tot_h);
+        }
     }
     named_sync(1, NTC);
-    uint8_t* z1 = buf + DATAB - S.n1;
+    uint8_t* z1 = arena + S.apos + ZPRE;
 #pragma unroll
     for (int j = 0; j < NP; ++j) {
         const uint32_t w = PW(j);
@@ -164,54 +192,55 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     constexpr int NWD2 = NB2 / 4;
 
     extern __shared__ __align__(1024) uint8_t smem[];
-    EncShared& S = *reinterpret_cast<EncShared*>(smem + NSTAGE * BUFB);
+    EncShared& S = *reinterpret_cast<EncShared*>(smem + SHARED_OFF);
+    uint8_t* const arena = smem + ARENA_OFF;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint64_t C = p.C;
+    const uint64_t full_chunks = p.n / CW;
 
     QConst qc = p.qc;
     if (MODE == MODE_NOA) qc = *p.qc_dev;
 
+    // ticket -> input stage s (compute warp 0 lane 0 only)
+    auto issue = [&](int s, unsigned long long t) {
+        S.in_c[s] = t;
+        if (t < full_chunks) {
+            fence_proxy_async();
+            mbar_arrive_tx(smem_u32(&S.full[s]), DATAB);
+            tma_load_2d(smem_u32(smem + s * DATAB), &tmap, 0, (int)(t * 128), smem_u32(&S.full[s]));
+        } else {
+            mbar_arrive(smem_u32(&S.full[s]));     // tail chunk (loaded by the compute warps) or end
+        }
+    };
+    unsigned long long next = 0;
     if (tid == 0) {
         if (smem_u32(smem) & 1023u) __trap();       // TMA SWIZZLE_128B needs 1024-byte alignment
-        for (int s = 0; s < NSTAGE; ++s) {
-            mbar_init(smem_u32(&S.full[s]), 1);
-            mbar_init(smem_u32(&S.ready[s]), 1);
+        for (int s = 0; s < NIN; ++s) mbar_init(smem_u32(&S.full[s]), 1);
+        for (int k = 0; k < NQ; ++k) {
+            mbar_init(smem_u32(&S.mq_full[k]), 1);
+            mbar_init(smem_u32(&S.mq_empty[k]), 1);
         }
+        S.head = 0;
+        S.tail = 0;
         fence_barrier_init();
+        prefetch_tmap(&tmap);
     }
     __syncthreads();
+    if (tid == 0) {
+        for (int s = 0; s < NIN; ++s) issue(s, atomicAdd(p.ticket, 1ull) - p.ticket_base);
+        next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+    }
 
     if (warp == NWC) {
         // =========================== IO warp ===========================
-        const uint64_t C = p.C;
-        const uint64_t full_chunks = p.n / CW;
-        unsigned long long next = 0;
-        auto issue = [&](int s, unsigned long long t) {
-            S.meta[s].c = t;
-            if (t < full_chunks) {
-                fence_proxy_async();
-                mbar_arrive_tx(smem_u32(&S.full[s]), DATAB);
-                tma_load_2d(smem_u32(smem + s * BUFB), &tmap, 0, (int)(t * 128), smem_u32(&S.full[s]));
-            } else {
-                mbar_arrive(smem_u32(&S.full[s]));       // tail chunk (compute loads it) or end
-            }
-        };
-        if (lane == 0) {
-            prefetch_tmap(&tmap);
-            for (int s = 0; s < NSTAGE; ++s) issue(s, atomicAdd(p.ticket, 1ull) - p.ticket_base);
-            next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-        }
-        __syncwarp();
         const uint64_t EP = (uint64_t)p.epoch << 48;
-        for (uint32_t it = 0;; ++it) {
-            const int s = it % NSTAGE;
-            const uint32_t ph = (it / NSTAGE) & 1u;
-            const uint64_t c = S.meta[s].c;
-            if (c >= C) break;
-            mbar_wait(smem_u32(&S.ready[s]), ph);
-            const uint32_t stored = S.meta[s].stored;
-            uint32_t start = S.meta[s].start;
-            const uint32_t israw = S.meta[s].raw;
-            // ---- decoupled look-back; the aggregate was published by compute ----
+        for (uint32_t k = 0;; ++k) {
+            const int slot = k % NQ;
+            mbar_wait(smem_u32(&S.mq_full[slot]), (k / NQ) & 1u);
+            const QEntry e = S.q[slot];
+            if (e.c >= C) break;
+            const uint64_t c = e.c;
+            // ---- decoupled look-back; compute published the aggregate ----
             uint64_t excl = 0;
             if (c > 0) {
                 int64_t look = (int64_t)c - 1;
@@ -223,6 +252,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                             const uint64_t d = ld_relaxed(&p.status[idx]);
                             flag = ((uint32_t)(d >> 48) == p.epoch) ? ((d >> 46) & 3u) : 0u;
                             if (flag) { val = d & LB_VAL; break; }
+                            __nanosleep(32);
                         }
                     }
                     const uint32_t pm = __ballot_sync(PFPL_FULL, flag == LB_P);
@@ -234,36 +264,36 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     excl += warp_sum64(val);
                     look -= 32;
                 }
-                if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + stored));
+                if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + e.stored));
             }
             const uint64_t dst = p.payload_off + excl;
             if (lane == 0) {
-                p.table[c] = stored;
-                if (c == C - 1) p.result[0] = dst + stored;
+                p.table[c] = e.stored;
+                if (c == C - 1) p.result[0] = dst + e.stored;
                 if (c == 0 && p.write_header) write_header(p.out, p, qc);
             }
-            uint8_t* buf = smem + s * BUFB;
-            if (dst + stored <= p.cap) {
-                if (israw) {
-                    // raw chunk (R17): stage the original bytes, aligned
-                    const uint8_t* src = (const uint8_t*)p.in + c * (uint64_t)kChunkBytes;
-                    for (uint32_t i = lane; i < stored / 16; i += 32) ((uint4*)buf)[i] = ldg_nc_v4(src + 16 * i);
-                    for (uint32_t i = (stored / 16) * 4 + lane; i < stored / 4; i += 32)
-                        ((uint32_t*)buf)[i] = ((const uint32_t*)src)[i];
+            if (dst + e.stored <= p.cap) {
+                const uint8_t* src = arena + e.start;
+                if (e.raw) {
+                    // raw chunk (R17): stage the original bytes in this chunk's
+                    // arena slice (always large enough: slice >= payload >= raw bytes)
+                    uint8_t* stg = arena + e.start;
+                    const uint8_t* g = (const uint8_t*)p.in + c * (uint64_t)kChunkBytes;
+                    for (uint32_t i = lane; i < e.stored / 16; i += 32) ((uint4*)stg)[i] = ldg_nc_v4(g + 16 * i);
+                    for (uint32_t i = (e.stored / 16) * 4 + lane; i < e.stored / 4; i += 32)
+                        ((uint32_t*)stg)[i] = ((const uint32_t*)g)[i];
                     __syncwarp();
-                    start = 0;
                 }
                 // 16-byte aligned stores for the body (coalesced even for
                 // unaligned compressed data), bytes for the head and tail
                 uint8_t* o = p.out + dst;
-                const uint8_t* src = buf + start;
                 const uint32_t mis = (uint32_t)((uintptr_t)o & 15u);
                 uint32_t head = (16u - mis) & 15u;
-                if (head > stored) head = stored;
-                const uint32_t body = (stored - head) >> 4;
+                if (head > e.stored) head = e.stored;
+                const uint32_t body = (e.stored - head) >> 4;
                 const uint32_t tail0 = head + (body << 4);
                 if ((uint32_t)lane < head) o[lane] = src[lane];
-                if ((uint32_t)lane < stored - tail0) o[tail0 + lane] = src[tail0 + lane];
+                if ((uint32_t)lane < e.stored - tail0) o[tail0 + lane] = src[tail0 + lane];
                 for (uint32_t j = lane; j < body; j += 32) {
                     const uint8_t* sp = src + head + (j << 4);
                     const uint32_t a = smem_u32(sp) & 3u;
@@ -280,11 +310,9 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             }
             __syncwarp();
             if (lane == 0) {
-                const unsigned long long t = next;
-                next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-                issue(s, t);
+                *(volatile uint32_t*)&S.tail = e.rend;     // release the arena slice
+                mbar_arrive(smem_u32(&S.mq_empty[slot]));
             }
-            __syncwarp();
         }
         return;
     }
@@ -293,13 +321,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     QF<T> q;
     q.load(qc);
     const bool raw = (qc.flags & HF_RAWWORDS) != 0;
-    for (uint32_t it = 0;; ++it) {
-        const int s = it % NSTAGE;
-        const uint32_t ph = (it / NSTAGE) & 1u;
-        mbar_wait(smem_u32(&S.full[s]), ph);
-        const uint64_t c = S.meta[s].c;
-        if (c >= p.C) break;
-        uint8_t* buf = smem + s * BUFB;
+    uint32_t it = 0;
+    for (;; ++it) {
+        const int s = it % NIN;
+        mbar_wait(smem_u32(&S.full[s]), (it / NIN) & 1u);
+        const uint64_t c = S.in_c[s];
+        if (c >= C) break;
+        const uint8_t* buf = smem + s * DATAB;
         const uint32_t m = (uint32_t)min((uint64_t)CW, p.n - c * (uint64_t)CW);
 
         // zero this thread's part of M1
@@ -360,7 +388,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const uint32_t oh = sizeof(W) == 8 ? __reduce_or_sync(PFPL_FULL, (uint32_t)((uint64_t)orv >> 32)) : 0u;
             if (lane == 0) S.wor[warp] = ((unsigned long long)oh << 32) | ol;
         }
-        named_sync(1, NTC);    // rows consumed, M1 zeroed, active planes known
+        named_sync(1, NTC);    // rows of stage s consumed, M1 zeroed, active planes known
+        if (tid == 0) {
+            // refill stage s with the prefetched ticket; prefetch the next one
+            const unsigned long long t = next;
+            next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+            issue(s, t);
+        }
         unsigned long long bor = 0;
 #pragma unroll
         for (int w = 0; w < NWC; ++w) bor |= S.wor[w];
@@ -368,22 +402,26 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
 
         // ---- bit shuffle + level-1 zero elimination (block-uniform tier) ----
         if (P == 0) {
-            if (tid == 0) S.n1 = 0;
+            if (tid == 0) {
+                S.n1 = 0;
+                reserve_arena(S, 0);
+            }
         } else if (B == 32 || P <= 32) {
-            if (P <= 4) rze1<T, 4, 0>(lo, hi, buf, S, tid, lane, warp);
-            else if (P <= 8) rze1<T, 8, 0>(lo, hi, buf, S, tid, lane, warp);
-            else if (P <= 16) rze1<T, 16, 0>(lo, hi, buf, S, tid, lane, warp);
-            else rze1<T, 32, 0>(lo, hi, buf, S, tid, lane, warp);
+            if (P <= 4) rze1<T, 4, 0>(lo, hi, arena, S, tid, lane, warp);
+            else if (P <= 8) rze1<T, 8, 0>(lo, hi, arena, S, tid, lane, warp);
+            else if (P <= 16) rze1<T, 16, 0>(lo, hi, arena, S, tid, lane, warp);
+            else rze1<T, 32, 0>(lo, hi, arena, S, tid, lane, warp);
         } else {
-            if (P <= 36) rze1<T, 32, 4>(lo, hi, buf, S, tid, lane, warp);
-            else if (P <= 40) rze1<T, 32, 8>(lo, hi, buf, S, tid, lane, warp);
-            else if (P <= 48) rze1<T, 32, 16>(lo, hi, buf, S, tid, lane, warp);
-            else rze1<T, 32, 32>(lo, hi, buf, S, tid, lane, warp);
+            if (P <= 36) rze1<T, 32, 4>(lo, hi, arena, S, tid, lane, warp);
+            else if (P <= 40) rze1<T, 32, 8>(lo, hi, arena, S, tid, lane, warp);
+            else if (P <= 48) rze1<T, 32, 16>(lo, hi, arena, S, tid, lane, warp);
+            else rze1<T, 32, 32>(lo, hi, arena, S, tid, lane, warp);
         }
         named_sync(1, NTC);    // Z1 and M1 complete
 
         // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 + Z2) ----
         const uint32_t n1 = S.n1;
+        uint8_t* const z1 = arena + S.apos + ZPRE;
         uint32_t n2 = 0;
         {
             uint32_t w2[NWD2], h2[NWD2];
@@ -413,8 +451,8 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 if (w < warp) base += v;
                 n2 += v;
             }
-            if (cnt2 && n1 + n2 <= (uint32_t)DATAB) {
-                uint8_t* z2 = buf + DATAB - n1 - n2;
+            if (cnt2) {
+                uint8_t* z2 = z1 - n2;
                 uint32_t o = base + inc - cnt2;
 #pragma unroll
                 for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
@@ -422,14 +460,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             if (NB2 == 16) ((uint16_t*)S.m2)[tid] = (uint16_t)bits2;
             else ((uint32_t*)S.m2)[tid] = bits2;
         }
-        fence_proxy_async();   // generic writes to the stage buffer before its next TMA refill
         if (warp != 0) {
             named_arrive(2, NTC);
             continue;
         }
         named_sync(2, NTC);
 
-        // ---- levels 3 and 4, size, raw decision (warp 0) ----
+        // ---- levels 3 and 4, size, raw decision, hand-off to the IO warp (warp 0) ----
         {
             const uint2 v = ((const uint2*)S.m2)[lane];
             const uint32_t pred = lane ? ((const uint32_t*)S.m2)[2 * lane - 1] : 0u;
@@ -444,29 +481,37 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const bool dif = m3 != pm3;
             const uint32_t M4 = __ballot_sync(PFPL_FULL, dif);
             const uint32_t n4 = __popc(M4);
+            uint8_t* z3 = z1 - n2 - n3;
+            scatter_word(z3, scatter_word(z3, inc3 - cnt3, v.x, h0), v.y, h1);
+            uint8_t* z4 = z3 - n4;
+            if (dif) z4[__popc(M4 & ((1u << lane) - 1u))] = (uint8_t)m3;
+            if (lane < 4) z4[lane - 4] = (uint8_t)(M4 >> (8 * lane));
             const uint32_t size = 4 + n4 + n3 + n2 + n1;
-            const bool fits = size <= (uint32_t)DATAB;
-            if (fits) {
-                uint8_t* z3 = buf + DATAB - n1 - n2 - n3;
-                scatter_word(z3, scatter_word(z3, inc3 - cnt3, v.x, h0), v.y, h1);
-                uint8_t* z4 = z3 - n4;
-                if (dif) z4[__popc(M4 & ((1u << lane) - 1u))] = (uint8_t)m3;
-                if (lane < 4) z4[lane - 4] = (uint8_t)(M4 >> (8 * lane));
-            }
             const uint32_t rawb = m * S_;
             const bool israw = size >= rawb;
             const uint32_t stored = israw ? rawb : size;
-            fence_proxy_async();
             __syncwarp();
             if (lane == 0) {
-                S.meta[s].stored = stored;
-                S.meta[s].start = fits ? (uint32_t)DATAB - size : 0u;
-                S.meta[s].raw = israw ? 1u : 0u;
                 const uint64_t EP = (uint64_t)p.epoch << 48;
                 st_relaxed(&p.status[c], EP | ((c == 0 ? LB_P : LB_A) << 46) | stored);
-                mbar_arrive(smem_u32(&S.ready[s]));
+                const int slot = it % NQ;
+                mbar_wait(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u);
+                QEntry& e = S.q[slot];
+                e.c = c;
+                e.stored = stored;
+                e.raw = israw ? 1u : 0u;
+                e.start = israw ? S.apos : (uint32_t)(z4 - 4 - arena);
+                e.rend = S.head;
+                mbar_arrive(smem_u32(&S.mq_full[slot]));
             }
         }
+    }
+    // end of work: tell the IO warp (the ring position `it` holds the first c >= C)
+    if (tid == 0) {
+        const int slot = it % NQ;
+        mbar_wait(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u);
+        S.q[slot].c = ~0ull;
+        mbar_arrive(smem_u32(&S.mq_full[slot]));
     }
 }
 
@@ -509,7 +554,7 @@ int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
 }
 
-int encode_stages() { return NSTAGE; }
+int encode_stages() { return NIN; }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
                                   const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
