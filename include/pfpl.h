@@ -134,6 +134,10 @@ int pfpl_decompress_chunks(const void* hdr_host, const uint32_t* table_host,
 /* ---- misc ---- */
 const char* pfpl_strerror(int status);
 int pfpl_last_cuda_error(void);
+/* If a kernel's bounded wait expired (a protocol error; the kernel traps and
+ * the call returns PFPL_ERR_CUDA), copies {site, block, thread, detail} to
+ * out4 and returns 1; otherwise returns 0. */
+int pfpl_watchdog_report(unsigned int* out4);
 /* Frees the calling thread's scratch for the current device. */
 int pfpl_release_scratch(void);
 /* Number of kernel launches issued by the library since load (for bench's

@@ -61,6 +61,7 @@ def lib():
             "pfpl_decompress_chunks": (i32, [vp, vp, u64, u64, vp, u64, vp, u64, vp]),
             "pfpl_strerror": (ctypes.c_char_p, [i32]),
             "pfpl_last_cuda_error": (i32, []),
+            "pfpl_watchdog_report": (i32, [ctypes.POINTER(ctypes.c_uint)]),
             "pfpl_release_scratch": (i32, []),
             "pfpl_launch_count": (u64, []),
             "pfpl_version": (ctypes.c_char_p, []),
@@ -77,6 +78,9 @@ def _check(st: int, what: str = ""):
         extra = ""
         if st == -6:
             extra = f"cudaError={lib().pfpl_last_cuda_error()}"
+            wd = (ctypes.c_uint * 4)()
+            if lib().pfpl_watchdog_report(wd):
+                extra += f" watchdog(site=0x{wd[0]:x}, block={wd[1]}, thread={wd[2]}, detail={wd[3]})"
         raise PFPLError(st, (what + " " + extra).strip())
 
 

@@ -41,6 +41,17 @@ struct Scratch {
 
 std::mutex g_mu;
 std::map<std::pair<int, void*>, Scratch*> g_scratch;
+unsigned int* g_wd_host = nullptr;     // mapped pinned watchdog report {site, block, thread, detail}
+unsigned int* g_wd_dev = nullptr;
+
+unsigned int* watchdog_ptr() {
+    if (!g_wd_host) {
+        if (cudaHostAlloc(&g_wd_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_wd_host = nullptr; return nullptr; }
+        memset(g_wd_host, 0, 64);
+        if (cudaHostGetDevicePointer(&g_wd_dev, g_wd_host, 0) != cudaSuccess) g_wd_dev = nullptr;
+    }
+    return g_wd_dev;
+}
 
 constexpr int kMinmaxBlocks = 592;
 
@@ -228,6 +239,7 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
     p.eps = eps;
     p.dtype = (uint32_t)dtype;
     p.bound = (uint32_t)bound;
+    p.wd = watchdog_ptr();
     const bool ms = (opts & PFPL_OPT_MS_RESIDUALS) != 0;
     const int grid = encode_grid(dtype, mode, ms, C);
     CK(launch_encode(dtype, mode, ms, p, grid, s));
@@ -329,6 +341,7 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     p.epoch = sc->epoch;
     p.qc = qc;
     p.err = err_dev;
+    p.wd = watchdog_ptr();
     const bool ms = (flags & HF_MS) != 0;
     const int grid = decode_grid(dtype, mode, ms, nchunks);
     CK(launch_decode(dtype, mode, ms, p, grid, s));
@@ -543,6 +556,12 @@ const char* pfpl_strerror(int st) {
 }
 
 int pfpl_last_cuda_error(void) { return g_last_cuda.load(); }
+
+int pfpl_watchdog_report(unsigned int* out4) {
+    if (!g_wd_host || !out4) return 0;
+    for (int i = 0; i < 4; ++i) out4[i] = ((volatile unsigned int*)g_wd_host)[i];
+    return out4[0] != 0;
+}
 
 int pfpl_release_scratch(void) {
     int dev = 0;

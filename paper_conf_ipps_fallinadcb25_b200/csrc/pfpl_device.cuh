@@ -143,8 +143,26 @@ template <> struct QF<float> {
         float vr = rb * c;
         float diff = fabsf(v - vr);
         bool ok = (fabsf(rb) < 4194304.0f) && (diff <= a);
-        int32_t bi = (int32_t)(f2u(t) - 0x4B400000u);
-        return ok ? zz(bi) : f2u(v);
+        // zigzag(rb) = 2|rb| - (rb < 0) = |2rb + 0.5| - 0.5, exact for |rb| < 2^22
+        const float w2 = __fmaf_rn(rb, 2.0f, 0.5f);
+        const uint32_t z = f2u(fabsf(w2) + 8388607.5f) - 0x4B000000u;
+        return ok ? z : f2u(v);
+    }
+    // biased word: abs_q(v) + 0x4B000000 (mod 2^32).  The bias cancels in the
+    // residuals q[i] - q[i-1], so the encoder can skip the integer subtraction:
+    // bits(|2rb + 0.5| + (2^23 - 0.5)) = 0x4B000000 + zigzag(rb) (two FMA-pipe ops)
+    __device__ __forceinline__ uint32_t abs_qb(float v) const {
+        float s = v * b;
+        float t = s + 12582912.0f;
+        float rb = t - 12582912.0f;
+        float vr = rb * c;
+        float diff = fabsf(v - vr);
+        bool ok = (fabsf(rb) < 4194304.0f) && (diff <= a);
+        const float w2 = __fmaf_rn(rb, 2.0f, 0.5f);
+        const uint32_t z = f2u(fabsf(w2) + 8388607.5f);
+        uint32_t rawb;
+        asm("mad.lo.u32 %0, %1, 1, 0x4B000000;" : "=r"(rawb) : "r"(f2u(v)));
+        return ok ? z : rawb;
     }
     __device__ __forceinline__ float abs_dq(uint32_t w) const {
         return w < 0x00800000u ? __int2float_rn(unzz(w)) * c : u2f(w);
@@ -196,6 +214,7 @@ template <> struct QF<double> {
         int64_t bi = (int64_t)(d2u(t) - 0x4338000000000000ull);
         return ok ? zz(bi) : d2u(v);
     }
+    __device__ __forceinline__ uint64_t abs_qb(double v) const { return abs_q(v); }
     __device__ __forceinline__ double abs_dq(uint64_t w) const {
         return w < 0x0010000000000000ull ? __ll2double_rn((long long)unzz(w)) * c : u2d(w);
     }
@@ -242,6 +261,18 @@ __device__ __forceinline__ typename Tr<T>::W quantize(const QF<T>& q, T v, bool 
     if (MODE == MODE_REL) return q.rel_q(v);
     return q.abs_q(v);
 }
+
+// encoder form: a word that differs from quantize() by a per-type constant
+// (QBIAS), which cancels in the delta coding
+template <typename T, int MODE>
+__device__ __forceinline__ typename Tr<T>::W quantize_b(const QF<T>& q, T v, bool raw) {
+    if (MODE == MODE_ABS || (MODE == MODE_NOA && !raw)) {
+        if (sizeof(T) == 4) return q.abs_qb(v);
+    }
+    return quantize<T, MODE>(q, v, raw);
+}
+template <typename T, int MODE> struct QBias { static constexpr uint64_t v = 0; };
+template <> struct QBias<float, MODE_ABS> { static constexpr uint64_t v = 0x4B000000u; };
 
 template <typename T, int MODE>
 __device__ __forceinline__ T dequantize(const QF<T>& q, typename Tr<T>::W w, bool raw);
@@ -346,6 +377,15 @@ template <int K> __device__ __forceinline__ void transpose_inv(uint32_t (&r)[32]
 __device__ __forceinline__ uint32_t nzbytes(uint32_t x) {
     return (((x & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | x) >> 7 & 0x01010101u;
 }
+// 0x80 in every non-zero byte of x
+__device__ __forceinline__ uint32_t nzmark(uint32_t x) {
+    return (((x & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | x) & 0x80808080u;
+}
+// H = nzmark(x): returns (lo, hi) of H * 0x02020202, i.e. lo byte k = number of
+// marked bytes below k (exclusive rank), hi byte 0 = number of marked bytes
+__device__ __forceinline__ uint64_t rankcount(uint32_t H) {
+    return (uint64_t)H * 0x02020202ull;
+}
 // gather the low bits of the 4 bytes of h (values 0/1) into a nibble
 __device__ __forceinline__ uint32_t nib(uint32_t h) { return (h * 0x10204080u) >> 28; }
 
@@ -416,6 +456,53 @@ __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
         "@P1 bra DONE;\n\t"
         "bra LAB_WAIT;\n"
         "DONE:\n\t}" ::"r"(a), "r"(parity) : "memory");
+}
+__device__ __forceinline__ bool mbar_test(uint32_t a, uint32_t parity) {
+    uint32_t r;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(r) : "r"(a), "r"(parity) : "memory");
+    return r != 0;
+}
+// ---- watchdog: every spin loop of the library is bounded in time.  On expiry
+// the site code, block and a detail word go to mapped host memory (readable
+// even after the context dies) and the kernel traps: a protocol bug becomes an
+// error (PFPL_ERR_CUDA) instead of a hung caller.
+static __device__ unsigned int* g_pfpl_wd;   // per TU; set from the kernel parameters
+constexpr uint64_t kWatchdogNs = 5000000000ull;   // 5 s
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+static __device__ __noinline__ void watchdog_fire(uint32_t site, uint32_t detail) {
+    unsigned int* h = g_pfpl_wd;
+    if (h) {
+        h[1] = blockIdx.x;
+        h[2] = threadIdx.x;
+        h[3] = detail;
+        __threadfence_system();
+        atomicExch(h, site);
+        __threadfence_system();
+    }
+    __trap();
+}
+__device__ __forceinline__ bool mbar_try(uint32_t a, uint32_t parity) {
+    uint32_t r;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(r) : "r"(a), "r"(parity) : "memory");
+    return r != 0;
+}
+__device__ __forceinline__ void mbar_wait_wd(uint32_t a, uint32_t parity, uint32_t site) {
+    if (mbar_try(a, parity)) return;
+    const uint64_t t0 = globaltimer();
+    for (uint32_t i = 1;; ++i) {
+        if (mbar_try(a, parity)) return;
+        if ((i & 63u) == 0 && globaltimer() - t0 > kWatchdogNs) watchdog_fire(site, parity);
+    }
 }
 __device__ __forceinline__ void fence_barrier_init() {
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");

@@ -33,8 +33,9 @@ constexpr int NIN = 2;               // input stages (TMA ring)
 constexpr int DATAB = 16384;         // bytes per chunk
 constexpr int ZPRE = 2352;           // >= 4 + 32 + 256 + 2048, multiple of 16
 constexpr int NQ = 8;                // IO queue depth
-constexpr int ARENA = 20800;         // circular payload arena (bytes, multiple of 16)
+constexpr int ARENA = 18752;         // circular payload arena (bytes, multiple of 16)
 
+// hand-off from the compute warps to the IO warp, one per chunk
 struct QEntry {
     unsigned long long c;
     uint32_t start, stored, raw, rend;
@@ -44,10 +45,8 @@ struct EncShared {
     uint8_t m1[2048];
     uint8_t m2[256];
     uint8_t wcnt[4][64];
-    uint16_t off[4][64];
-    unsigned long long wor[4];
-    uint32_t scan[4];
-    uint32_t n1, apos, head, tail;
+    uint32_t scan2[4];               // level-2 warp totals
+    uint32_t head, tail;
     unsigned long long in_c[NIN];
     QEntry q[NQ];
     unsigned long long full[NIN], mq_full[NQ], mq_empty[NQ];
@@ -82,6 +81,14 @@ __device__ __forceinline__ uint32_t scatter_word(uint8_t* z, uint32_t o, uint32_
     if (hh & 0x1000000u) z[o + ((incl >> 16) & 0xFFu)] = (uint8_t)(w >> 24);
     return o + (incl >> 24);
 }
+// same with the marker at bit 7 (H = nzmark(w)); ranks from one IMAD.WIDE
+__device__ __forceinline__ void scatter_marked(uint8_t* z, uint32_t o, uint32_t w, uint32_t H) {
+    const uint32_t rk = (uint32_t)rankcount(H);          // byte k = rank of byte k
+    if (H & 0x80u) z[o] = (uint8_t)w;
+    if (H & 0x8000u) z[o + __byte_perm(rk, 0, 0x4441)] = (uint8_t)(w >> 8);
+    if (H & 0x800000u) z[o + __byte_perm(rk, 0, 0x4442)] = (uint8_t)(w >> 16);
+    if (H & 0x80000000u) z[o + (rk >> 24)] = (uint8_t)(w >> 24);
+}
 
 // ---------------------------------------------------------------------------
 // bit shuffle + level-1 zero-byte elimination for one chunk.
@@ -94,94 +101,102 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
     return *(const volatile uint32_t*)p;
 }
 
-// reserve ZPRE + n1 bytes of the arena (compute warp 0, lane 0); waits only if
-// the IO warp lags by more than the arena's capacity
-__device__ __forceinline__ void reserve_arena(EncShared& S, uint32_t n1) {
-    const uint32_t R = (ZPRE + n1 + 15u) & ~15u;
+// Arena slice for a chunk with n1 Z1 bytes: every compute warp derives the same
+// position from S.head (advanced by warp 0 only after the Z1 scatter) and waits
+// only if the IO warp lags by more than the arena's capacity.
+__device__ __forceinline__ uint32_t slice_bytes(uint32_t n1) { return (ZPRE + n1 + 15u) & ~15u; }
+__device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
+    const uint32_t R = slice_bytes(n1);
     uint32_t head = S.head;
     const uint32_t p0 = head % ARENA;
-    if (p0 + R > (uint32_t)ARENA) head += ARENA - p0;      // do not wrap a slice
-    while (head + R - ld_volatile_u32(&S.tail) > (uint32_t)ARENA) __nanosleep(64);
-    S.apos = head % ARENA;
-    S.head = head + R;
+    if (p0 + R > (uint32_t)ARENA) head += ARENA - p0;      // a slice never wraps
+    if (lane == 0 && head + R - ld_volatile_u32(&S.tail) > (uint32_t)ARENA) {
+        const uint64_t t0 = globaltimer();
+        while (head + R - ld_volatile_u32(&S.tail) > (uint32_t)ARENA) {
+            if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x13, head);
+            __nanosleep(64);
+        }
+    }
+    __syncwarp();
+    return head;                                            // monotone byte counter
 }
 
+// ---- level-1 phase A: transpose in place, per-plane counts, packed warp scans.
+// KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
+// Plane word j holds bit b_j of the thread's 32 residuals (b_j = j, or 32+j-KL).
+// Writes this warp's full row of per-plane counts (zero above its tier).
 template <typename T, int KL, int KH>
-__device__ __forceinline__ void rze1(uint32_t (&lo)[32], uint32_t (&hi)[32], uint8_t* arena,
-                                     EncShared& S, int tid, int lane, int warp) {
-    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NW = Tr<T>::NW, NTC = Tr<T>::NT;
-    constexpr int NP = KL + KH, NG = NP / 4;
-    transpose_fwd<KL>(lo);
+__device__ __forceinline__ void rze1_count(uint32_t (&lo)[32], uint32_t (&hi)[32], EncShared& S,
+                                           int lane, int warp, uint64_t wor, uint32_t (&ex)[16]) {
+    constexpr int B = Tr<T>::B;
+    constexpr int NG = (KL + KH) / 4;
+    if constexpr (KL > 0) transpose_fwd<KL>(lo);
     if constexpr (KH > 0) transpose_fwd<KH>(hi);
     auto PW = [&](int j) -> uint32_t { return j < KL ? lo[j] : hi[j - KL]; };
-    // per-plane non-zero byte counts (0..4), 4 planes per word, 8 bits each
-    uint32_t ex[NG];
 #pragma unroll
     for (int g = 0; g < NG; ++g) {
-        uint32_t v = 0;
-#pragma unroll
-        for (int i = 0; i < 4; ++i) v += ((nzbytes(PW(4 * g + i)) * 0x01010101u) >> 24) << (8 * i);
-        uint32_t inc = v;
-        if (__any_sync(PFPL_FULL, v != 0)) inc = warp_incl_scan(v, lane);
-        ex[g] = inc - v;
         const int b0 = 4 * g < KL ? 4 * g : 32 + 4 * g - KL;
+        uint32_t inc = 0, v = 0;
+        if (wor & (0xFull << b0)) {          // skip groups empty in this whole warp
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+                v = __byte_perm(v, (uint32_t)(rankcount(nzmark(PW(4 * g + i))) >> 32),
+                                i == 0 ? 0x3214 : i == 1 ? 0x3240 : i == 2 ? 0x3410 : 0x4210);
+            inc = warp_incl_scan(v, lane);
+        }
+        ex[g] = inc - v;
         if (lane == 31) *(uint32_t*)&S.wcnt[warp][b0] = inc;
     }
-    named_sync(1, NTC);
-    if (warp == 0) {
-        // plane order = decreasing bit index; lane l owns bit l (and 32+l)
-        uint32_t wl[NW], wh[NW], tl = 0, th = 0;
+    if (lane == 31) {
 #pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            wl[w] = lane < KL ? S.wcnt[w][lane] : 0u;
-            wh[w] = lane < KH ? S.wcnt[w][32 + lane] : 0u;
-            tl += wl[w];
-            th += wh[w];
-        }
-        uint32_t sl = tl, sh = th;   // inclusive suffix sums over lanes
+        for (int b0 = KL; b0 < 32; b0 += 4) *(uint32_t*)&S.wcnt[warp][b0] = 0u;
 #pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            const uint32_t a = __shfl_down_sync(PFPL_FULL, sl, d);
-            const uint32_t b = KH > 0 ? __shfl_down_sync(PFPL_FULL, sh, d) : 0u;
-            if (lane + d < 32) { sl += a; sh += b; }
-        }
-        const uint32_t tot_h = KH > 0 ? __shfl_sync(PFPL_FULL, sh, 0) : 0u;
-        const uint32_t tot_l = __shfl_sync(PFPL_FULL, sl, 0);
-        uint32_t run = tot_h + sl - tl;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            if (lane < KL) S.off[w][lane] = (uint16_t)run;
-            run += wl[w];
-        }
-        if (KH > 0) {
-            run = sh - th;
-#pragma unroll
-            for (int w = 0; w < NW; ++w) {
-                if (lane < KH) S.off[w][32 + lane] = (uint16_t)run;
-                run += wh[w];
-            }
-        }
-        if (lane == 0) {
-            S.n1 = tot_l + tot_h;
-            reserve_arena(S, tot_l + tot_h);
-        }
-    }
-    named_sync(1, NTC);
-    uint8_t* z1 = arena + S.apos + ZPRE;
-#pragma unroll
-    for (int j = 0; j < NP; ++j) {
-        const uint32_t w = PW(j);
-        if (!__any_sync(PFPL_FULL, w != 0)) continue;          // warp-uniform skip of empty planes
-        const int b = j < KL ? j : 32 + j - KL;
-        const int pl = B - 1 - b;
-        const uint32_t hj = nzbytes(w);
-        const uint32_t o = S.off[warp][b] + ((ex[j / 4] >> (8 * (j % 4))) & 0xFFu);
-        scatter_word(z1, o, w, hj);
-        const uint32_t nb = nib(hj);
-        const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
-        if (!(lane & 1)) S.m1[pl * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
+        for (int b0 = 32 + KH; b0 < B; b0 += 4) *(uint32_t*)&S.wcnt[warp][b0] = 0u;
     }
 }
+
+// ---- level-1 phase B: scatter the non-zero bytes of this thread's plane words
+// to Z1 (plane-major order, R13) and its M1 nibbles; offl/offh = this warp's
+// Z1 offset of the segment of bit `lane` / `32+lane`.
+template <typename T, int KL, int KH>
+__device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uint32_t (&hi)[32],
+                                             uint8_t* z1, uint8_t* m1, int tid, int lane,
+                                             uint64_t wor, const uint32_t (&ex)[16],
+                                             uint32_t offl, uint32_t offh) {
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW;
+    constexpr int NP = KL + KH;
+#pragma unroll
+    for (int j = 0; j < NP; ++j) {
+        const uint32_t w = j < KL ? lo[j] : hi[j - KL];
+        const int b = j < KL ? j : 32 + j - KL;
+        if (!((wor >> b) & 1u)) continue;                       // plane empty in this warp
+        if (!__any_sync(PFPL_FULL, w != 0)) continue;
+        const int pl = B - 1 - b;
+        const uint32_t H = nzmark(w);
+        const uint32_t o = __shfl_sync(PFPL_FULL, j < KL ? offl : offh, b & 31) +
+                           __byte_perm(ex[j / 4], 0, 0x4440 + (j % 4));
+        scatter_marked(z1, o, w, H);
+        const uint32_t nb = nib(H >> 7);
+        const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
+        if (!(lane & 1)) m1[pl * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
+    }
+}
+
+#define PFPL_TIER_DISPATCH(FN, ...)                                                     \
+    do {                                                                                \
+        if (P == 0) FN<T, 0, 0>(__VA_ARGS__);                                           \
+        else if (B == 32 || P <= 32) {                                                  \
+            if (P <= 4) FN<T, 4, 0>(__VA_ARGS__);                                       \
+            else if (P <= 8) FN<T, 8, 0>(__VA_ARGS__);                                  \
+            else if (P <= 16) FN<T, 16, 0>(__VA_ARGS__);                                \
+            else FN<T, 32, 0>(__VA_ARGS__);                                             \
+        } else {                                                                        \
+            if (P <= 36) FN<T, 32, 4>(__VA_ARGS__);                                     \
+            else if (P <= 40) FN<T, 32, 8>(__VA_ARGS__);                                \
+            else if (P <= 48) FN<T, 32, 16>(__VA_ARGS__);                               \
+            else FN<T, 32, 32>(__VA_ARGS__);                                            \
+        }                                                                               \
+    } while (0)
 
 template <typename T, int MODE, bool MSR>
 __global__ void __launch_bounds__(Tr<T>::NT + 32, 4)
@@ -214,6 +229,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     };
     unsigned long long next = 0;
     if (tid == 0) {
+        g_pfpl_wd = p.wd;
         if (smem_u32(smem) & 1023u) __trap();       // TMA SWIZZLE_128B needs 1024-byte alignment
         for (int s = 0; s < NIN; ++s) mbar_init(smem_u32(&S.full[s]), 1);
         for (int k = 0; k < NQ; ++k) {
@@ -236,11 +252,21 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         const uint64_t EP = (uint64_t)p.epoch << 48;
         for (uint32_t k = 0;; ++k) {
             const int slot = k % NQ;
-            mbar_wait(smem_u32(&S.mq_full[slot]), (k / NQ) & 1u);
+            mbar_wait_wd(smem_u32(&S.mq_full[slot]), (k / NQ) & 1u, 0x11);
             const QEntry e = S.q[slot];
             if (e.c >= C) break;
             const uint64_t c = e.c;
-            // ---- decoupled look-back; compute published the aggregate ----
+            // lag behind the compute warps by up to one entry (bounded, so a slice
+            // that fills the arena cannot deadlock): by then the predecessors of
+            // chunk c have almost always published their aggregates
+            {
+                const uint32_t nb = smem_u32(&S.mq_full[(k + 1) % NQ]);
+                const uint32_t np = ((k + 1) / NQ) & 1u;
+                for (int tries = 0; tries < 16 && !mbar_test(nb, np); ++tries) __nanosleep(256);
+            }
+            const uint32_t stored = e.stored, start = e.start;
+            const bool israw = e.raw != 0;
+            // ---- decoupled look-back ----
             uint64_t excl = 0;
             if (c > 0) {
                 int64_t look = (int64_t)c - 1;
@@ -248,11 +274,15 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     const int64_t idx = look - lane;
                     uint64_t val = 0, flag = LB_P;
                     if (idx >= 0) {
-                        for (;;) {
+                        // the predecessor may still be in flight: back off so the
+                        // polling does not steal issue slots from the compute warps
+                        const uint64_t t0 = globaltimer();
+                        for (uint32_t ns = 256;; ns = ns < 8192 ? 2 * ns : ns) {
                             const uint64_t d = ld_relaxed(&p.status[idx]);
                             flag = ((uint32_t)(d >> 48) == p.epoch) ? ((d >> 46) & 3u) : 0u;
                             if (flag) { val = d & LB_VAL; break; }
-                            __nanosleep(32);
+                            if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x12, (uint32_t)idx);
+                            __nanosleep(ns);
                         }
                     }
                     const uint32_t pm = __ballot_sync(PFPL_FULL, flag == LB_P);
@@ -264,23 +294,23 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     excl += warp_sum64(val);
                     look -= 32;
                 }
-                if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + e.stored));
+                if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + stored));
             }
             const uint64_t dst = p.payload_off + excl;
             if (lane == 0) {
-                p.table[c] = e.stored;
-                if (c == C - 1) p.result[0] = dst + e.stored;
+                p.table[c] = stored;
+                if (c == C - 1) p.result[0] = dst + stored;
                 if (c == 0 && p.write_header) write_header(p.out, p, qc);
             }
-            if (dst + e.stored <= p.cap) {
-                const uint8_t* src = arena + e.start;
-                if (e.raw) {
+            if (dst + stored <= p.cap) {
+                const uint8_t* src = arena + start;
+                if (israw) {
                     // raw chunk (R17): stage the original bytes in this chunk's
                     // arena slice (always large enough: slice >= payload >= raw bytes)
-                    uint8_t* stg = arena + e.start;
+                    uint8_t* stg = arena + start;
                     const uint8_t* g = (const uint8_t*)p.in + c * (uint64_t)kChunkBytes;
-                    for (uint32_t i = lane; i < e.stored / 16; i += 32) ((uint4*)stg)[i] = ldg_nc_v4(g + 16 * i);
-                    for (uint32_t i = (e.stored / 16) * 4 + lane; i < e.stored / 4; i += 32)
+                    for (uint32_t i = lane; i < stored / 16; i += 32) ((uint4*)stg)[i] = ldg_nc_v4(g + 16 * i);
+                    for (uint32_t i = (stored / 16) * 4 + lane; i < stored / 4; i += 32)
                         ((uint32_t*)stg)[i] = ((const uint32_t*)g)[i];
                     __syncwarp();
                 }
@@ -289,11 +319,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 uint8_t* o = p.out + dst;
                 const uint32_t mis = (uint32_t)((uintptr_t)o & 15u);
                 uint32_t head = (16u - mis) & 15u;
-                if (head > e.stored) head = e.stored;
-                const uint32_t body = (e.stored - head) >> 4;
+                if (head > stored) head = stored;
+                const uint32_t body = (stored - head) >> 4;
                 const uint32_t tail0 = head + (body << 4);
                 if ((uint32_t)lane < head) o[lane] = src[lane];
-                if ((uint32_t)lane < e.stored - tail0) o[tail0 + lane] = src[tail0 + lane];
+                if ((uint32_t)lane < stored - tail0) o[tail0 + lane] = src[tail0 + lane];
                 for (uint32_t j = lane; j < body; j += 32) {
                     const uint8_t* sp = src + head + (j << 4);
                     const uint32_t a = smem_u32(sp) & 3u;
@@ -321,25 +351,30 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     QF<T> q;
     q.load(qc);
     const bool raw = (qc.flags & HF_RAWWORDS) != 0;
+    // bias of quantize_b(): only the f32 ABS/NOA bin path is biased
+    const uint64_t qbias = (sizeof(T) == 4 && (MODE == MODE_ABS || (MODE == MODE_NOA && !raw)))
+                               ? 0x4B000000ull : 0ull;
     uint32_t it = 0;
     for (;; ++it) {
         const int s = it % NIN;
-        mbar_wait(smem_u32(&S.full[s]), (it / NIN) & 1u);
+        mbar_wait_wd(smem_u32(&S.full[s]), (it / NIN) & 1u, 0x14);
         const uint64_t c = S.in_c[s];
         if (c >= C) break;
         const uint8_t* buf = smem + s * DATAB;
+        uint8_t* const m1 = S.m1;
         const uint32_t m = (uint32_t)min((uint64_t)CW, p.n - c * (uint64_t)CW);
 
         // zero this thread's part of M1
 #pragma unroll
         for (int i = 0; i < 2048 / 16 / NTC; ++i)
-            ((uint4*)S.m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
+            ((uint4*)m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
 
         // ---- quantize + verify, delta, residual code ----
         uint32_t lo[32], hi[32];
         W orv = 0;
         {
-            W qprev = 0;
+            // biased words (quantize_b): q + bias; the bias cancels in q[i] - q[i-1]
+            W qprev = (W)qbias;
             if (m == CW) {
                 if (tid > 0) {
                     T pv;
@@ -350,7 +385,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         const int r = 2 * tid - 1;
                         pv = *(const T*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 8);
                     }
-                    qprev = quantize<T, MODE>(q, pv, raw);
+                    qprev = quantize_b<T, MODE>(q, pv, raw);
                 }
 #pragma unroll
                 for (int i = 0; i < 2 * S_; ++i) {
@@ -360,7 +395,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     memcpy(x, &v, 16);
 #pragma unroll
                     for (int k = 0; k < 16 / S_; ++k) {
-                        const W qw = quantize<T, MODE>(q, x[k], raw);
+                        const W qw = quantize_b<T, MODE>(q, x[k], raw);
                         const W r2 = rcode<MSR>((W)(qw - qprev));
                         qprev = qw;
                         orv |= r2;
@@ -371,10 +406,10 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             } else {
                 // tail chunk: plain loads; R12 pads with the last value -> zero residuals
                 const T* src = (const T*)p.in + c * (uint64_t)CW;
-                if (tid > 0) qprev = quantize<T, MODE>(q, src[min(32 * tid - 1, (int)m - 1)], raw);
+                if (tid > 0) qprev = quantize_b<T, MODE>(q, src[min(32 * tid - 1, (int)m - 1)], raw);
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
-                    const W qw = quantize<T, MODE>(q, src[min(32 * tid + i, (int)m - 1)], raw);
+                    const W qw = quantize_b<T, MODE>(q, src[min(32 * tid + i, (int)m - 1)], raw);
                     const W r2 = rcode<MSR>((W)(qw - qprev));
                     qprev = qw;
                     orv |= r2;
@@ -383,71 +418,87 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 }
             }
         }
-        {
-            const uint32_t ol = __reduce_or_sync(PFPL_FULL, (uint32_t)orv);
-            const uint32_t oh = sizeof(W) == 8 ? __reduce_or_sync(PFPL_FULL, (uint32_t)((uint64_t)orv >> 32)) : 0u;
-            if (lane == 0) S.wor[warp] = ((unsigned long long)oh << 32) | ol;
-        }
-        named_sync(1, NTC);    // rows of stage s consumed, M1 zeroed, active planes known
+        // this warp's active planes (warp-uniform tier; other warps may differ)
+        const uint32_t ol = __reduce_or_sync(PFPL_FULL, (uint32_t)orv);
+        const uint32_t oh = sizeof(W) == 8 ? __reduce_or_sync(PFPL_FULL, (uint32_t)((uint64_t)orv >> 32)) : 0u;
+        const uint64_t wor = ((uint64_t)oh << 32) | ol;
+        const int P = wor ? 64 - __clzll((long long)wor) : 0;
+
+        // ---- bit shuffle + level-1 zero elimination ----
+        uint32_t ex[16];
+        PFPL_TIER_DISPATCH(rze1_count, lo, hi, S, lane, warp, wor, ex);
+        named_sync(1, NTC);    // counts visible; every row of stage s consumed
         if (tid == 0) {
             // refill stage s with the prefetched ticket; prefetch the next one
             const unsigned long long t = next;
             next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
             issue(s, t);
         }
-        unsigned long long bor = 0;
+        // Z1 offsets of this warp's segments: planes in decreasing bit order,
+        // then warps (lane l owns bit l and 32+l)
+        uint32_t offl, offh, n1, head;
+        {
+            uint32_t myl = 0, myh = 0, tl = 0, th = 0;
 #pragma unroll
-        for (int w = 0; w < NWC; ++w) bor |= S.wor[w];
-        const int P = bor ? 64 - __clzll((long long)bor) : 0;
-
-        // ---- bit shuffle + level-1 zero elimination (block-uniform tier) ----
-        if (P == 0) {
-            if (tid == 0) {
-                S.n1 = 0;
-                reserve_arena(S, 0);
+            for (int w = 0; w < NWC; ++w) {
+                const uint32_t a = S.wcnt[w][lane];
+                const uint32_t b = B == 64 ? S.wcnt[w][32 + lane] : 0u;
+                if (w < warp) { myl += a; myh += b; }
+                tl += a;
+                th += b;
             }
-        } else if (B == 32 || P <= 32) {
-            if (P <= 4) rze1<T, 4, 0>(lo, hi, arena, S, tid, lane, warp);
-            else if (P <= 8) rze1<T, 8, 0>(lo, hi, arena, S, tid, lane, warp);
-            else if (P <= 16) rze1<T, 16, 0>(lo, hi, arena, S, tid, lane, warp);
-            else rze1<T, 32, 0>(lo, hi, arena, S, tid, lane, warp);
-        } else {
-            if (P <= 36) rze1<T, 32, 4>(lo, hi, arena, S, tid, lane, warp);
-            else if (P <= 40) rze1<T, 32, 8>(lo, hi, arena, S, tid, lane, warp);
-            else if (P <= 48) rze1<T, 32, 16>(lo, hi, arena, S, tid, lane, warp);
-            else rze1<T, 32, 32>(lo, hi, arena, S, tid, lane, warp);
+            uint32_t sl = tl, sh = th;   // inclusive suffix sums over lanes
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t a = __shfl_down_sync(PFPL_FULL, sl, d);
+                const uint32_t b = B == 64 ? __shfl_down_sync(PFPL_FULL, sh, d) : 0u;
+                if (lane + d < 32) { sl += a; sh += b; }
+            }
+            const uint32_t tot_h = B == 64 ? __shfl_sync(PFPL_FULL, sh, 0) : 0u;
+            const uint32_t tot_l = __shfl_sync(PFPL_FULL, sl, 0);
+            offl = tot_h + sl - tl + myl;
+            offh = sh - th + myh;
+            n1 = tot_l + tot_h;
+            head = slice_start(S, n1, lane);
         }
+        uint8_t* const z1 = arena + head % ARENA + ZPRE;
+        PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
         named_sync(1, NTC);    // Z1 and M1 complete
+        if (tid == 0) S.head = head + slice_bytes(n1);
 
-        // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 + Z2) ----
-        const uint32_t n1 = S.n1;
-        uint8_t* const z1 = arena + S.apos + ZPRE;
-        uint32_t n2 = 0;
+        // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 + Z2), P:131 ----
+        const int slot = it % NQ;
         {
             uint32_t w2[NWD2], h2[NWD2];
-            const uint32_t* m1w = (const uint32_t*)S.m1;
+            const uint32_t* m1w = (const uint32_t*)m1;
 #pragma unroll
             for (int i = 0; i < NWD2; i += 4) {
                 const uint4 v = *(const uint4*)(m1w + NWD2 * tid + i);
                 w2[i] = v.x; w2[i + 1] = v.y; w2[i + 2] = v.z; w2[i + 3] = v.w;
             }
             const uint32_t pred = tid ? m1w[NWD2 * tid - 1] : 0u;
-            uint32_t bits2 = 0;
+            uint32_t bits2 = 0, any = pred;
 #pragma unroll
-            for (int i = 0; i < NWD2; ++i) {
-                const uint32_t pw = i ? w2[i - 1] : pred;
-                h2[i] = nzbytes(w2[i] ^ __funnelshift_l(pw, w2[i], 8));
-                bits2 |= nib(h2[i]) << (4 * i);
+            for (int i = 0; i < NWD2; ++i) any |= w2[i];
+            if (__any_sync(PFPL_FULL, any != 0)) {           // M1 of inactive planes is all zero
+#pragma unroll
+                for (int i = 0; i < NWD2; ++i) {
+                    const uint32_t pw = i ? w2[i - 1] : pred;
+                    h2[i] = nzbytes(w2[i] ^ __funnelshift_l(pw, w2[i], 8));
+                    bits2 |= nib(h2[i]) << (4 * i);
+                }
             }
+            if (NB2 == 16) ((uint16_t*)S.m2)[tid] = (uint16_t)bits2;
+            else ((uint32_t*)S.m2)[tid] = bits2;
             const uint32_t cnt2 = __popc(bits2);
             uint32_t inc = cnt2;
             if (__any_sync(PFPL_FULL, cnt2 != 0)) inc = warp_incl_scan(cnt2, lane);
-            if (lane == 31) S.scan[warp] = inc;
-            named_sync(1, NTC);
-            uint32_t base = 0;
+            if (lane == 31) S.scan2[warp] = inc;
+            named_sync(1, NTC);    // M2 complete, level-2 warp totals visible
+            uint32_t base = 0, n2 = 0;
 #pragma unroll
             for (int w = 0; w < NWC; ++w) {
-                const uint32_t v = S.scan[w];
+                const uint32_t v = S.scan2[w];
                 if (w < warp) base += v;
                 n2 += v;
             }
@@ -457,20 +508,14 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
 #pragma unroll
                 for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
             }
-            if (NB2 == 16) ((uint16_t*)S.m2)[tid] = (uint16_t)bits2;
-            else ((uint32_t*)S.m2)[tid] = bits2;
-        }
-        if (warp != 0) {
-            named_arrive(2, NTC);
-            continue;
-        }
-        named_sync(2, NTC);
 
-        // ---- levels 3 and 4, size, raw decision, hand-off to the IO warp (warp 0) ----
-        {
+            // ---- levels 3 and 4 on the 256-byte M2, size, raw decision,
+            // aggregate, hand-off: one duty warp, rotating so no warp is always late ----
+            if (warp != (int)(it % NWC)) continue;
             const uint2 v = ((const uint2*)S.m2)[lane];
-            const uint32_t pred = lane ? ((const uint32_t*)S.m2)[2 * lane - 1] : 0u;
-            const uint32_t h0 = nzbytes(v.x ^ __funnelshift_l(pred, v.x, 8));
+            uint32_t pm2 = __shfl_up_sync(PFPL_FULL, v.y, 1);
+            if (lane == 0) pm2 = 0;
+            const uint32_t h0 = nzbytes(v.x ^ __funnelshift_l(pm2, v.x, 8));
             const uint32_t h1 = nzbytes(v.y ^ __funnelshift_l(v.x, v.y, 8));
             const uint32_t m3 = nib(h0) | (nib(h1) << 4);
             const uint32_t cnt3 = __popc(m3);
@@ -494,22 +539,21 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             if (lane == 0) {
                 const uint64_t EP = (uint64_t)p.epoch << 48;
                 st_relaxed(&p.status[c], EP | ((c == 0 ? LB_P : LB_A) << 46) | stored);
-                const int slot = it % NQ;
-                mbar_wait(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u);
+                mbar_wait_wd(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u, 0x15);
                 QEntry& e = S.q[slot];
                 e.c = c;
                 e.stored = stored;
                 e.raw = israw ? 1u : 0u;
-                e.start = israw ? S.apos : (uint32_t)(z4 - 4 - arena);
-                e.rend = S.head;
+                e.start = israw ? head % ARENA : (uint32_t)(z4 - 4 - arena);
+                e.rend = head + slice_bytes(n1);
                 mbar_arrive(smem_u32(&S.mq_full[slot]));
             }
         }
     }
-    // end of work: tell the IO warp (the ring position `it` holds the first c >= C)
+    // end of work: tell the IO warp (queue position `it` gets a terminal entry)
     if (tid == 0) {
         const int slot = it % NQ;
-        mbar_wait(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u);
+        mbar_wait_wd(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u, 0x16);
         S.q[slot].c = ~0ull;
         mbar_arrive(smem_u32(&S.mq_full[slot]));
     }

@@ -44,6 +44,7 @@ struct EncParams {
     uint64_t n_total;        // header n
     double eps;              // header eps
     uint32_t dtype, bound;   // header bytes 5, 6
+    unsigned int* wd;        // watchdog report (mapped host memory) or null
 };
 
 struct DecParams {
@@ -59,6 +60,7 @@ struct DecParams {
     uint32_t epoch;
     QConst qc;               // a/b/c as in QConst; decoder uses eb2 (ABS/NOA) or w (REL)
     int* err;                // set to PFPL_ERR_CORRUPT on malformed chunks
+    unsigned int* wd;        // watchdog report (mapped host memory) or null
 };
 
 // kernel launchers (pfpl_kernels.cu)
