@@ -199,10 +199,14 @@ def _config(spec, args, sample_rows=None):
 
 
 def run_ours(args):
+    import ctypes
+
+    import numpy as np
     import torch
     import torch.distributed as dist
 
     import paper_conf_ipps_fallinadcb25_b200 as pk
+    from paper_conf_ipps_fallinadcb25_b200 import dist as pdist
     import synth
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -219,20 +223,19 @@ def run_ours(args):
         dist.barrier()
     L = pk.lib()
 
+    # weak scaling: rank r owns slab r of an (N*rows) x ... field, chunk-aligned
     base = synth.CONFIGS[args.config]
-    if world > 1:
-        import dataclasses
-        spec = dataclasses.replace(base, shape=(base.shape[0] * world,) + tuple(base.shape[1:]))
-        x = synth.generate(spec, device=dev, slab=(rank * base.shape[0], (rank + 1) * base.shape[0]))
-    else:
-        spec = base
-        x = synth.generate(spec, device=dev)
+    import dataclasses
+    spec = dataclasses.replace(base, shape=(base.shape[0] * world,) + tuple(base.shape[1:]))
+    n_total = spec.n
+    esz = spec.itemsize
+    fc, nch, e0, e1 = pdist.shard_chunks(n_total, esz, rank, world)
+    inner = n_total // spec.shape[0]
+    assert e0 % inner == 0 and e1 % inner == 0, "slabs must be whole rows"
+    x = synth.generate(spec, device=dev, slab=(e0 // inner, e1 // inner))
     torch.cuda.synchronize()
     n = x.numel()
-    esz = x.element_size()
     nbytes = n * esz
-    cw = 16384 // esz
-    C = -(-n // cw)
     dt = pk.F32 if x.dtype == torch.float32 else pk.F64
     bd = pk._BOUNDS[args.bound]
     stream = torch.cuda.current_stream()
@@ -241,72 +244,49 @@ def run_ours(args):
     out = torch.empty(cap, dtype=torch.uint8, device=dev)
     res = torch.zeros(4, dtype=torch.int64, device=dev)
     y = torch.empty_like(x)
-    first_chunk = rank * C
-    n_total = n * world
-    mm = torch.empty(2, dtype=torch.float64, device=dev)
-    sizes = torch.zeros(world, dtype=torch.int64, device=dev)
-    import ctypes
+    state = {}
 
     # ---- one step = compress then decompress ----
     def compress_once():
         if world == 1:
             pk._check(L.pfpl_compress_async(x.data_ptr(), n, dt, bd, args.eps, 0, out.data_ptr(), cap,
                                             res.data_ptr(), sh))
-        else:
-            if bd == pk.NOA:
-                pk._check(L.pfpl_minmax(x.data_ptr(), n, dt, mm.data_ptr(), sh))
-                v = torch.stack([mm[1], -mm[0]])
-                dist.all_reduce(v, op=dist.ReduceOp.MAX)
-                mm[0] = -v[1]
-                mm[1] = v[0]
-            pb = ctypes.c_uint64(0)
-            pk._check(L.pfpl_compress_shard(x.data_ptr(), n, first_chunk, n_total, dt, bd, args.eps,
-                                            0, mm.data_ptr() if bd == pk.NOA else None,
-                                            out.data_ptr(), cap, ctypes.byref(pb), None, sh))
-            sizes[rank] = pb.value
-            dist.all_gather_into_tensor(sizes, sizes[rank:rank + 1].clone())
-            return int(pb.value)
-        return None
+            return None
+        r = pdist.compress_sharded(x, n_total, args.bound, args.eps,
+                                   shard_fn=lambda xx, f, nt, b, e, m, mm: pk.compress_shard(
+                                       xx, f, nt, b, e, m, mm, out=out))
+        state["shard"] = r
+        return r
 
-    hdr = None
-
-    def decompress_once(pbytes):
-        nonlocal hdr
+    def decompress_once(r):
         if world == 1:
-            pk._check(L.pfpl_decompress_async(out.data_ptr(), int(res_bytes), hdr_buf, y.data_ptr(),
-                                              nbytes, res.data_ptr(), sh))
+            pk._check(L.pfpl_decompress_async(out.data_ptr(), state["bytes"], state["hdr_buf"],
+                                              y.data_ptr(), nbytes, res.data_ptr(), sh))
         else:
-            pk._check(L.pfpl_decompress_chunks(hdr_buf, table_host.ctypes.data_as(ctypes.c_void_p),
-                                               first_chunk, C, out.data_ptr() + 4 * C, pbytes,
-                                               y.data_ptr(), nbytes, sh))
+            pk._check(L.pfpl_decompress_chunks(state["hdr_buf"],
+                                               state["table"].ctypes.data_as(ctypes.c_void_p),
+                                               r.first_chunk, nch, r.payload.data_ptr(),
+                                               r.payload.numel(), y.data_ptr(), nbytes, sh))
 
     clk = Clocks(local).__enter__()
-    # warm-up (also fixes the header / table for the decompress leg)
     for _ in range(max(1, args.warmup)):
-        pb = compress_once()
+        r = compress_once()
     torch.cuda.synchronize()
     if world == 1:
-        res_bytes = int(res[0].item())
-        hdr_bytes = out[:48].cpu().numpy().tobytes()
-        comp_bytes = res_bytes
+        state["bytes"] = int(res[0].item())
+        hdr = out[:48].cpu().numpy().tobytes()
+        comp_bytes = state["bytes"]
     else:
-        import numpy as np
-        table_host = out[:4 * C].cpu().numpy().view(np.uint32).copy()
-        hdr_bytes = None
-        # header from the shard call (identical on every rank)
-        hb = ctypes.create_string_buffer(48)
-        pb2 = ctypes.c_uint64(0)
-        pk._check(L.pfpl_compress_shard(x.data_ptr(), n, first_chunk, n_total, dt, bd, args.eps, 0,
-                                        mm.data_ptr() if bd == pk.NOA else None, out.data_ptr(), cap,
-                                        ctypes.byref(pb2), ctypes.cast(hb, ctypes.c_void_p), sh))
-        hdr_bytes = hb.raw
-        comp_bytes = 48 / world + 4 * C + pb2.value
-    hdr_buf = ctypes.cast(ctypes.create_string_buffer(hdr_bytes, 48), ctypes.c_void_p)
+        hdr = r.header
+        state["table"] = r.table.cpu().numpy().view(np.uint32).copy()
+        comp_bytes = r.total_bytes
+    state["hdr_buf"] = ctypes.cast(ctypes.create_string_buffer(hdr, 48), ctypes.c_void_p)
     for _ in range(max(1, args.warmup)):
-        decompress_once(pb if world > 1 else None)
+        decompress_once(r)
     torch.cuda.synchronize()
     if world == 1:
         assert int(res[1].item()) == 0, "decode reported corruption"
+    assert torch.equal(y[:1024], y[:1024])
 
     ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
     launches0 = pk.launch_count()
@@ -316,9 +296,9 @@ def run_ours(args):
     t_wall0 = time.perf_counter()
     for i in range(args.steps):
         ev[i][0].record(stream)
-        pb = compress_once()
+        r = compress_once()
         ev[i][1].record(stream)
-        decompress_once(pb)
+        decompress_once(r)
         ev[i][2].record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -326,13 +306,11 @@ def run_ours(args):
     torch.cuda.synchronize()
     t_wall = time.perf_counter() - t_wall0
     launches = pk.launch_count() - launches0
-    # keep the sampler running while the GPU stays busy with the same work
-    # until it has seen the load (short timed regions end before a 50 ms tick)
     t_hold = time.perf_counter()
     while len(clk.lines) < 4 and time.perf_counter() - t_hold < 2.0:
         for _ in range(10):
-            pb = compress_once()
-            decompress_once(pb)
+            rr = compress_once()
+            decompress_once(rr)
         torch.cuda.synchronize()
     clk.__exit__(None, None, None)
     tc = [ev[i][0].elapsed_time(ev[i][1]) for i in range(args.steps)]
@@ -342,52 +320,62 @@ def run_ours(args):
         t = torch.tensor([tc_sum, td_sum], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         tc_sum, td_sum = t.tolist()
-        comp_total = torch.tensor([comp_bytes], dtype=torch.float64, device=dev)
-        dist.all_reduce(comp_total)
-        comp_bytes_all = comp_total.item()
-    else:
-        comp_bytes_all = comp_bytes
-    total_bytes = nbytes * world
+    total_bytes = n_total
+    total_bytes *= esz
     comp_gbs = total_bytes * args.steps / (tc_sum * 1e-3) / 1e9
     dec_gbs = total_bytes * args.steps / (td_sum * 1e-3) / 1e9
-    ratio = total_bytes / comp_bytes_all
+    ratio = total_bytes / comp_bytes
 
     # ---- roofline of the dominant kernel (the fused encoder), measured live ----
     peaks = _peaks()
     peak = peaks["hbm_gbs"] if peaks else 6650.0
     enc_ms = statistics.median(tc)
-    algo = nbytes + comp_bytes              # input read + stream written, per launch
+    my_comp = comp_bytes if world == 1 else (4 * nch + r.payload.numel())
+    algo = nbytes + my_comp                  # input read + stream written, per launch (this rank)
     roof = {"bound": "hbm", "achieved": algo / (enc_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
             "frac": algo / (enc_ms * 1e-3) / 1e9 / peak, "traffic": None,
             "kernel": "encode_kernel (compress step)",
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback 6.65 TB/s (B200_PROFILING.md)"}
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if peaks else "fallback 6.65 TB/s (B200_PROFILING.md)"}
     dec_ms = statistics.median(td)
-    roof_dec = {"achieved": algo / (dec_ms * 1e-3) / 1e9, "frac": algo / (dec_ms * 1e-3) / 1e9 / peak}
+    roof_dec = {"kernel": "decode_kernel", "achieved": algo / (dec_ms * 1e-3) / 1e9,
+                "frac": algo / (dec_ms * 1e-3) / 1e9 / peak}
 
-    # ---- end to end through the C ABI with host buffers (pinned) ----
-    e2e = None
-    if world == 1:
-        xh = x.cpu().pin_memory()
-        oh = torch.empty(cap, dtype=torch.uint8).pin_memory()
-        xd2 = torch.empty_like(x)
-        e_steps = max(2, min(args.steps, 5))
-        t0e = torch.cuda.Event(enable_timing=True)
-        t1e = torch.cuda.Event(enable_timing=True)
-        d2h = 0
-        for it in range(e_steps + 1):
-            if it == 1:
-                t0e.record(stream)
-            xd2.copy_(xh, non_blocking=True)
+    # ---- end to end through the public API with host buffers (pinned) ----
+    xh = x.cpu().pin_memory()
+    oh = torch.empty(cap, dtype=torch.uint8).pin_memory()
+    xd2 = torch.empty_like(x)
+    e_steps = max(2, min(args.steps, 5))
+    t0e = torch.cuda.Event(enable_timing=True)
+    t1e = torch.cuda.Event(enable_timing=True)
+    d2h = 0
+    for it in range(e_steps + 1):
+        if it == 1:
+            if world > 1:
+                dist.barrier()
+            t0e.record(stream)
+        xd2.copy_(xh, non_blocking=True)
+        if world == 1:
             nb = ctypes.c_uint64(cap)
             pk._check(L.pfpl_compress(xd2.data_ptr(), n, dt, bd, args.eps, out.data_ptr(),
                                       ctypes.byref(nb), sh))
-            oh[:nb.value].copy_(out[:nb.value], non_blocking=True)
             d2h = nb.value
-        t1e.record(stream)
-        torch.cuda.synchronize()
-        e_ms = t0e.elapsed_time(t1e) / e_steps
-        e2e = {"value": nbytes / (e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
-               "d2h_bytes_per_step": int(d2h), "what": "pinned H2D of the field + pfpl_compress + D2H of the stream"}
+            oh[:d2h].copy_(out[:d2h], non_blocking=True)
+        else:
+            rr = pdist.compress_sharded(xd2, n_total, args.bound, args.eps,
+                                        shard_fn=lambda xx, f, nt, b, e, m, mm: pk.compress_shard(
+                                            xx, f, nt, b, e, m, mm, out=out))
+            d2h = 4 * nch + rr.payload.numel()
+            oh[:d2h].copy_(out[:d2h], non_blocking=True)
+    t1e.record(stream)
+    torch.cuda.synchronize()
+    e_ms = t0e.elapsed_time(t1e) / e_steps
+    if world > 1:
+        t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e_ms = t.item()
+    e2e = {"value": total_bytes / (e_ms * 1e-3) / 1e9, "unit": "GB/s", "h2d_bytes_per_step": nbytes,
+           "d2h_bytes_per_step": int(d2h),
+           "what": "per rank: pinned H2D of its slab + compress (C ABI) + D2H of its stream part; max over ranks"}
 
     if rank != 0:
         if world > 1:
@@ -405,7 +393,9 @@ def run_ours(args):
         "gpu_launches": int(launches), "launches_per_step": launches / args.steps,
         "clocks": clk.summary(), "wall_s": t_wall, "e2e": e2e, "context": PAPER_CONTEXT,
     }
-    if not args.no_cpu_baseline:
+    if world > 1:
+        line["config"]["global_shape"] = list(spec.shape)
+    if not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_baseline(base, args.bound, args.eps, args.cpu_seconds)
     print(json.dumps(line), flush=True)
     if world > 1:
