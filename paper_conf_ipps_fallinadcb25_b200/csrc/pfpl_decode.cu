@@ -1,155 +1,188 @@
 // pfpl_decode.cu -- fused PFPL chunk decoder for sm_100a.
 //
-// The exact inverse of pfpl_encode.cu: chunk offsets by a single-pass
-// look-back over the stored size table ("the decoder computes a prefix
-// sum over the stored chunk sizes"), payload staged once in shared memory,
-// repeated-byte levels 4->2 and the zero-byte level rebuilt top-down with
-// block-wide prefix sums over bitmap popcounts, inverse bit-plane
-// transpose in registers, negabinary -> two's complement and the
-// delta decoder's block-wide inclusive scan (the decoder bottleneck
-// P:302/P:342), dequantize and 16-byte coalesced stores.
-#include <type_traits>
+// The exact inverse of pfpl_encode.cu ("Decompression employs the inverse
+// of these transformations in the opposite order").  Persistent,
+// warp-specialised CTAs:
+//
+//   IO warp                                   compute warps (4 for f32, 2 for f64)
+//   -------                                   ------------------------------------
+//   ticket c; chunk offset = prefix of the     wait full[s]; repeat levels 4 -> 2
+//   stored sizes by a look-back over the rebuilt top-down with popcount
+//   size table, which never waits:     prefix ranks -- every warp
+//   all sizes are known; validate; load the    derives M3/M2 itself, no barrier;
+//   payload into stage s with cp.async.bulk    zero level: gather the plane
+//   (2-stage ring)                             words from Z1, inverse bit shuffle in
+//                                              registers, negabinary^-1 and
+//                                              the delta decoder's inclusive scan
+//                                              (the decode bottleneck P:302),
+//                                              dequantize into swizzled
+//                                              rows; one thread stores the chunk with
+//                                              a TMA 2-D tensor store
+#include <cuda.h>
 #include "pfpl_device.cuh"
 
 namespace pfpl {
 
-template <typename T> struct DecGeom {
-    static constexpr int NT = Tr<T>::NT, S = Tr<T>::S;
-    static constexpr int ROWB = 32 * S + 16;
-    static constexpr int OUTB = NT * ROWB;
-    static constexpr int PAYB = 16 + 2352 + 16384 + 64;
-    static constexpr int BUF = OUTB > PAYB ? OUTB : PAYB;
+constexpr int DIN = 2;                 // payload stages
+constexpr int DSTG = 16448;            // payload stage bytes (16384 + alignment slack)
+constexpr int DOUT_OFF = DIN * DSTG;   // swizzled output staging (1024-aligned below)
+
+struct DecMeta {
+    unsigned long long c;
+    uint32_t size, delta, bad, pad;
 };
 
-__device__ __forceinline__ void set_err(int* err) { atomicExch(err, -4); }
+struct DecShared {
+    uint8_t m1[2048];
+    uint8_t act[128];                  // non-zero flag per 16-byte M1 segment
+    uint8_t wcnt[4][64];
+    unsigned long long wtot[4];        // per-warp totals of the delta scan
+    DecMeta meta[DIN];
+    unsigned long long full[DIN], empty[DIN];
+};
+constexpr int DOUT = (DOUT_OFF + 1023) & ~1023;
+constexpr int DSH_OFF = DOUT + 16384;
+constexpr int DEC_SMEM = DSH_OFF + (int)sizeof(DecShared);
+static_assert(DEC_SMEM <= 57344, "4 CTAs per SM need <= 56 KiB of shared memory each");
 
-// level-1 inverse: gather this thread's plane words from Z1 (plane-major order)
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t mbar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(dst), "l"(src), "r"(bytes), "r"(mbar) : "memory");
+}
+__device__ __forceinline__ void tma_store_2d(const void* tmap, int x, int y, uint32_t src) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                 ::"l"(tmap), "r"(x), "r"(y), "r"(src) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// ---- level 1 inverse, phase A: nibbles of this thread's plane words, counts
 template <typename T, int KL, int KH>
-__device__ __forceinline__ void rze1_dec(uint32_t (&lo)[32], uint32_t (&hi)[32], const uint8_t* z1,
-                                         const uint8_t* s_m1, uint8_t (*s_wcnt)[64],
-                                         uint16_t (*s_off)[64], uint32_t* s_n1, int tid,
-                                         int lane, int warp) {
-    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NW = Tr<T>::NW;
+__device__ __forceinline__ void dec1_count(const uint8_t* m1, DecShared& S, int tid, int lane,
+                                          int warp, uint32_t (&nb)[64], uint32_t (&ex)[16]) {
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW;
     constexpr int NP = KL + KH, NG = NP / 4;
-    uint32_t nb[NP];
 #pragma unroll
     for (int j = 0; j < NP; ++j) {
         const int b = j < KL ? j : 32 + j - KL;
         const int pl = B - 1 - b;
-        nb[j] = (s_m1[pl * (CW / 64) + (tid >> 1)] >> (4 * (tid & 1))) & 0xFu;
+        nb[j] = (m1[pl * (CW / 64) + (tid >> 1)] >> (4 * (tid & 1))) & 0xFu;
     }
-    uint32_t ex[NG];
 #pragma unroll
     for (int g = 0; g < NG; ++g) {
         uint32_t v = 0;
 #pragma unroll
         for (int i = 0; i < 4; ++i) v |= (uint32_t)__popc(nb[4 * g + i]) << (8 * i);
-        const uint32_t inc = warp_incl_scan(v, lane);
+        uint32_t inc = 0;
+        if (__any_sync(PFPL_FULL, v != 0)) inc = warp_incl_scan(v, lane);
         ex[g] = inc - v;
         const int b0 = 4 * g < KL ? 4 * g : 32 + 4 * g - KL;
-        if (lane == 31) *(uint32_t*)&s_wcnt[warp][b0] = inc;
+        if (lane == 31) *(uint32_t*)&S.wcnt[warp][b0] = inc;
     }
-    __syncthreads();
-    if (warp == 0) {
-        uint32_t wl[NW], wh[NW], tl = 0, th = 0;
+    if (lane == 31) {
 #pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            wl[w] = lane < KL ? s_wcnt[w][lane] : 0u;
-            wh[w] = lane < KH ? s_wcnt[w][32 + lane] : 0u;
-            tl += wl[w];
-            th += wh[w];
-        }
-        uint32_t sl = tl, sh = th;
+        for (int b0 = KL; b0 < 32; b0 += 4) *(uint32_t*)&S.wcnt[warp][b0] = 0u;
 #pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-            uint32_t a = __shfl_down_sync(PFPL_FULL, sl, d);
-            uint32_t b = __shfl_down_sync(PFPL_FULL, sh, d);
-            if (lane + d < 32) { sl += a; sh += b; }
-        }
-        const uint32_t tot_h = __shfl_sync(PFPL_FULL, sh, 0);
-        const uint32_t tot_l = __shfl_sync(PFPL_FULL, sl, 0);
-        uint32_t run = tot_h + sl - tl;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            if (lane < KL) s_off[w][lane] = (uint16_t)run;
-            run += wl[w];
-        }
-        run = sh - th;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            if (lane < KH) s_off[w][32 + lane] = (uint16_t)run;
-            run += wh[w];
-        }
-        if (lane == 0) *s_n1 = tot_l + tot_h;
+        for (int b0 = 32 + KH; b0 < B; b0 += 4) *(uint32_t*)&S.wcnt[warp][b0] = 0u;
     }
-    __syncthreads();
-    uint32_t pw[NP];
+}
+
+// ---- level 1 inverse, phase B: gather the plane words from Z1, inverse transpose
+template <typename T, int KL, int KH>
+__device__ __forceinline__ void dec1_gather(uint32_t (&lo)[32], uint32_t (&hi)[32], const uint8_t* z1,
+                                           int lane, const uint32_t (&nb)[64],
+                                           const uint32_t (&ex)[16], uint32_t offl, uint32_t offh) {
+    constexpr int NP = KL + KH;
 #pragma unroll
     for (int j = 0; j < NP; ++j) {
         const int b = j < KL ? j : 32 + j - KL;
-        const uint32_t o = s_off[warp][b] + ((ex[j / 4] >> (8 * (j % 4))) & 0xFFu);
+        const uint32_t o = __shfl_sync(PFPL_FULL, j < KL ? offl : offh, b & 31) +
+                           __byte_perm(ex[j / 4], 0, 0x4440 + (j % 4));
         const uint32_t n = nb[j];
         uint32_t w = 0, r = o;
         if (n & 1u) w |= (uint32_t)z1[r++];
         if (n & 2u) w |= (uint32_t)z1[r++] << 8;
         if (n & 4u) w |= (uint32_t)z1[r++] << 16;
         if (n & 8u) w |= (uint32_t)z1[r] << 24;
-        pw[j] = w;
+        if (j < KL) lo[j] = w; else hi[j - KL] = w;
     }
+    if constexpr (KL > 0) transpose_inv<KL>(lo);
+    else {
 #pragma unroll
-    for (int j = 0; j < KL; ++j) lo[j] = pw[j];
-    transpose_inv<KL>(lo);
-    if constexpr (KH > 0) {
-#pragma unroll
-        for (int j = 0; j < KH; ++j) hi[j] = pw[KL + j];
-        transpose_inv<KH>(hi);
-    } else {
+        for (int i = 0; i < 32; ++i) lo[i] = 0;
+    }
+    if constexpr (KH > 0) transpose_inv<KH>(hi);
+    else {
 #pragma unroll
         for (int i = 0; i < 32; ++i) hi[i] = 0;
     }
 }
 
+#define PFPL_DEC_TIER(FN, ...)                                                          \
+    do {                                                                                \
+        if (P == 0) FN<T, 0, 0>(__VA_ARGS__);                                           \
+        else if (B == 32 || P <= 32) {                                                  \
+            if (P <= 4) FN<T, 4, 0>(__VA_ARGS__);                                       \
+            else if (P <= 8) FN<T, 8, 0>(__VA_ARGS__);                                  \
+            else if (P <= 16) FN<T, 16, 0>(__VA_ARGS__);                                \
+            else FN<T, 32, 0>(__VA_ARGS__);                                             \
+        } else {                                                                        \
+            if (P <= 36) FN<T, 32, 4>(__VA_ARGS__);                                     \
+            else if (P <= 40) FN<T, 32, 8>(__VA_ARGS__);                                \
+            else if (P <= 48) FN<T, 32, 16>(__VA_ARGS__);                               \
+            else FN<T, 32, 32>(__VA_ARGS__);                                            \
+        }                                                                               \
+    } while (0)
+
+__device__ __forceinline__ void set_err(int* err) { atomicExch(err, -4); }
+
 template <typename T, int MODE, bool MSR>
-__global__ void __launch_bounds__(Tr<T>::NT) decode_kernel(const DecParams p) {
+__global__ void __launch_bounds__(Tr<T>::NT + 32, 4)
+decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
-    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NT = Tr<T>::NT, NW = Tr<T>::NW, S = Tr<T>::S;
-    constexpr int ROWB = DecGeom<T>::ROWB;
-    constexpr int NB2 = 2048 / NT;
-    constexpr int NWD2 = NB2 / 4;
-    typedef typename std::conditional<B == 32, uint32_t, unsigned long long>::type ActT;
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;
+    constexpr int NB2 = 2048 / NTC;          // M1 bytes per compute thread (16 or 32)
 
-    __shared__ __align__(16) uint8_t s_buf[DecGeom<T>::BUF];
-    __shared__ __align__(16) uint8_t s_m1[2048];
-    __shared__ __align__(16) uint8_t s_m2[256];
-    __shared__ __align__(16) uint8_t s_wcnt[NW][64];
-    __shared__ __align__(16) uint16_t s_off[NW][64];
-    __shared__ W s_scanw[NW];
-    __shared__ uint32_t s_scan[NW];
-    __shared__ ActT s_act[NW];
-    __shared__ unsigned long long s_c, s_poff;
-    __shared__ uint32_t s_size, s_delta, s_n1, s_n3, s_n4, s_bad;
-
+    extern __shared__ __align__(1024) uint8_t smem[];
+    DecShared& S = *reinterpret_cast<DecShared*>(smem + DSH_OFF);
+    uint8_t* const stage_out = smem + DOUT;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    QF<T> q;
-    q.load(p.qc);
-    const bool raw = (p.qc.flags & HF_RAWWORDS) != 0;
+    const uint64_t C = p.C;
 
-    for (;;) {
-        if (tid == 0) s_c = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-        if (tid < NW) s_act[tid] = 0;
-        __syncthreads();
-        const uint64_t c = s_c;
-        if (c >= p.C) break;
-        const uint32_t m = (uint32_t)min((uint64_t)CW, p.n - c * (uint64_t)CW);
-        const uint32_t rawb = m * S;
+    if (tid == 0) {
+        g_pfpl_wd = p.wd;
+        if (smem_u32(smem) & 1023u) __trap();
+        for (int s = 0; s < DIN; ++s) {
+            mbar_init(smem_u32(&S.full[s]), 1);
+            mbar_init(smem_u32(&S.empty[s]), 1);
+        }
+        fence_barrier_init();
+        prefetch_tmap(&tmap);
+    }
+    __syncthreads();
 
-        // ---- d1: chunk offset = prefix of stored sizes (look-back) ----
-        if (warp == 0) {
+    if (warp == NWC) {
+        // =========================== IO warp ===========================
+        const uint64_t EP = (uint64_t)p.epoch << 48;
+        unsigned long long tnext = 0;
+        if (lane == 0) tnext = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+        for (uint32_t it = 0;; ++it) {
+            const int s = it % DIN;
+            const unsigned long long c = __shfl_sync(PFPL_FULL, tnext, 0);
+            if (lane == 0) tnext = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+            mbar_wait_wd(smem_u32(&S.empty[s]), ((it / DIN) & 1u) ^ 1u, 0x21);
+            if (c >= C) {
+                if (lane == 0) {
+                    S.meta[s].c = c;
+                    mbar_arrive(smem_u32(&S.full[s]));
+                }
+                break;
+            }
+            // d1: offset = sum of the stored sizes before c (look-back)
             const uint32_t size = p.table[c];
-            const uint64_t EP = (uint64_t)p.epoch << 48;
             uint64_t excl = 0;
-            int64_t look = (int64_t)c - 1;
-            while (look >= 0) {
+            for (int64_t look = (int64_t)c - 1; look >= 0; look -= 32) {
                 const int64_t idx = look - lane;
                 uint64_t val = 0;
                 bool isP = false;
@@ -165,158 +198,194 @@ __global__ void __launch_bounds__(Tr<T>::NT) decode_kernel(const DecParams p) {
                     break;
                 }
                 excl += warp_sum64(val);
-                look -= 32;
             }
+            const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
+            const uint32_t rawb = m * S_;
+            uint32_t bad = 0;
+            if (size > rawb || excl + size > p.in_bytes) bad = 1;
+            if (c == C - 1 && excl + size != p.in_bytes) bad = 1;
+            if (size < 4 && size != rawb) bad = 1;
+            if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | ((excl + size) & LB_VAL));
+            // stage the payload: 16-byte aligned superset by one bulk copy (never
+            // past the last 16-byte boundary of the stream), the rest by the lanes
+            uint8_t* stg = smem + s * DSTG;
+            const uint8_t* g = p.in + excl;
+            const uint32_t delta = (uint32_t)((uintptr_t)g & 15u);
+            const uint8_t* a0 = g - delta;
+            const uint8_t* want = g + size;
+            const uint8_t* a1 = (const uint8_t*)(((uintptr_t)want + 15u) & ~(uintptr_t)15u);
+            const uint8_t* lim = (const uint8_t*)((uintptr_t)(p.in + p.in_bytes) & ~(uintptr_t)15u);
+            if (a1 > lim) a1 = lim;
+            if (a1 < a0) a1 = a0;
+            const uint32_t bulk = bad ? 0u : (uint32_t)(a1 - a0);
+            if (!bad)
+                for (const uint8_t* q = a1 + lane; q < want; q += 32) stg[q - a0] = *q;
+            __syncwarp();
             if (lane == 0) {
-                st_relaxed(&p.status[c], EP | (LB_P << 46) | ((excl + size) & LB_VAL));
-                uint32_t bad = 0;
-                if (size > rawb || excl + size > p.in_bytes) bad = 1;
-                if (c == p.C - 1 && excl + size != p.in_bytes) bad = 1;
-                if (size < 4 && size != rawb) bad = 1;
-                s_bad = bad;
-                s_size = size;
-                s_poff = excl;
-                s_delta = (uint32_t)((uintptr_t)(p.in + excl) & 15u);
-            }
-        }
-        __syncthreads();
-        if (s_bad) {
-            if (tid == 0) set_err(p.err);
-            continue;
-        }
-        const uint32_t size = s_size, delta = s_delta;
-        // ---- stage the payload: 16-byte aligned blocks, guarded at the ends ----
-        {
-            const uint8_t* g0 = p.in + s_poff - delta;          // 16-byte aligned
-            const uint8_t* lo_ok = p.in;
-            const uint8_t* hi_ok = p.in + p.in_bytes;
-            const uint32_t nblk = (delta + size + 15) >> 4;
-            for (uint32_t j = tid; j < nblk; j += NT) {
-                const uint8_t* a = g0 + 16 * j;
-                if (a >= lo_ok && a + 16 <= hi_ok) {
-                    ((uint4*)s_buf)[j] = ldg_nc_v4(a);
+                DecMeta& md = S.meta[s];
+                md.c = c;
+                md.size = size;
+                md.delta = delta;
+                md.bad = bad;
+                if (bulk) {
+                    mbar_arrive_tx(smem_u32(&S.full[s]), bulk);
+                    bulk_g2s(smem_u32(stg), a0, bulk, smem_u32(&S.full[s]));
                 } else {
-                    for (int k = 0; k < 16; ++k)
-                        s_buf[16 * j + k] = (a + k >= lo_ok && a + k < hi_ok) ? a[k] : (uint8_t)0;
+                    mbar_arrive(smem_u32(&S.full[s]));
                 }
             }
         }
-        __syncthreads();
+        return;
+    }
+
+    // ============================ compute warps ============================
+    QF<T> q;
+    q.load(p.qc);
+    const bool raw = (p.qc.flags & HF_RAWWORDS) != 0;
+    for (uint32_t it = 0;; ++it) {
+        const int s = it % DIN;
+        mbar_wait_wd(smem_u32(&S.full[s]), (it / DIN) & 1u, 0x22);
+        const DecMeta md = S.meta[s];
+        const uint64_t c = md.c;
+        if (c >= C) break;
+        const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
+        const uint8_t* pay = smem + s * DSTG + md.delta;
         uint8_t* const dstc = (uint8_t*)p.out + c * (uint64_t)kChunkBytes;
-        if (size == rawb) {
+        if (md.bad) {
+            named_sync(1, NTC);
+            if (tid == 0) { set_err(p.err); mbar_arrive(smem_u32(&S.empty[s])); }
+            continue;
+        }
+        if (md.size == m * S_) {
             // raw chunk: the stored bytes are the original values
-            {
-                const uint8_t* sp = s_buf + delta;
-                for (uint32_t j = tid; j < rawb / 4; j += NT) {
-                    const uint32_t a = (uint32_t)__cvta_generic_to_shared(sp + 4 * j) & 3u;
-                    const uint32_t* sw = (const uint32_t*)(sp + 4 * j - a);
-                    ((uint32_t*)dstc)[j] = __funnelshift_r(sw[0], sw[1], 8u * a);
-                }
+            const uint32_t nw = md.size / 4;
+            for (uint32_t j = tid; j < nw; j += NTC) {
+                const uint32_t a = smem_u32(pay + 4 * j) & 3u;
+                const uint32_t* sw = (const uint32_t*)(pay + 4 * j - a);
+                ((uint32_t*)dstc)[j] = __funnelshift_r(sw[0], sw[1], 8u * a);
             }
+            named_sync(1, NTC);
+            if (tid == 0) mbar_arrive(smem_u32(&S.empty[s]));
             continue;
         }
-        const uint8_t* const pay = s_buf + delta;
 
-        // ---- levels 4 and 3 (warp 0): M4 -> M3 -> M2 ----
-        if (warp == 0) {
-            const uint32_t M4 = (uint32_t)pay[0] | ((uint32_t)pay[1] << 8) | ((uint32_t)pay[2] << 16) | ((uint32_t)pay[3] << 24);
-            const uint32_t n4 = __popc(M4);
-            const uint8_t* z4 = pay + 4;
-            const uint32_t c4 = __popc(M4 & (lane == 31 ? 0xFFFFFFFFu : ((2u << lane) - 1u)));
-            const uint32_t m3 = c4 ? z4[c4 - 1] : 0u;
-            const uint32_t cnt3 = __popc(m3);
-            const uint32_t inc3 = warp_incl_scan(cnt3, lane);
-            const uint32_t n3 = __shfl_sync(PFPL_FULL, inc3, 31);
-            const uint8_t* z3 = z4 + n4;
-            const uint32_t e3 = inc3 - cnt3;
-            uint32_t w0 = 0, w1 = 0;
+        // ---- levels 4 -> 3 -> 2, derived by every warp (no barrier) ----
+        const uint32_t M4 = (uint32_t)pay[0] | ((uint32_t)pay[1] << 8) | ((uint32_t)pay[2] << 16) |
+                            ((uint32_t)pay[3] << 24);
+        const uint32_t n4 = __popc(M4);
+        const uint8_t* z4 = pay + 4;
+        const uint32_t c4 = __popc(M4 & (lane == 31 ? 0xFFFFFFFFu : ((2u << lane) - 1u)));
+        const uint32_t m3 = c4 ? z4[c4 - 1] : 0u;              // M3 byte `lane`
+        const uint32_t cnt3 = __popc(m3);
+        const uint32_t inc3 = warp_incl_scan(cnt3, lane);
+        const uint32_t n3 = __shfl_sync(PFPL_FULL, inc3, 31);
+        const uint8_t* z3 = z4 + n4;
+        uint32_t m2lo = 0, m2hi = 0;                            // M2 bytes 8*lane .. 8*lane+7
 #pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                const uint32_t cj = e3 + __popc(m3 & ((2u << j) - 1u));
-                const uint32_t bv = cj ? z3[cj - 1] : 0u;
-                if (j < 4) w0 |= bv << (8 * j); else w1 |= bv << (8 * (j - 4));
-            }
-            ((uint2*)s_m2)[lane] = make_uint2(w0, w1);
-            if (lane == 0) { s_n4 = n4; s_n3 = n3; }
+        for (int j = 0; j < 8; ++j) {
+            const uint32_t cj = inc3 - cnt3 + __popc(m3 & ((2u << j) - 1u));
+            const uint32_t bv = cj ? z3[cj - 1] : 0u;
+            if (j < 4) m2lo |= bv << (8 * j); else m2hi |= bv << (8 * (j - 4));
         }
-        __syncthreads();
-
-        // ---- level 2 (all threads): M2 -> M1, and active (plane, warp) segments ----
+        const uint32_t pc2 = __popc(m2lo) + __popc(m2hi);
+        const uint32_t inc2 = warp_incl_scan(pc2, lane);
+        const uint32_t n2 = __shfl_sync(PFPL_FULL, inc2, 31);
+        const uint8_t* z2 = z3 + n3;
+        // ---- level 2 -> M1: thread t owns M1 bytes [NB2*t, NB2*t + NB2) ----
         {
-            const uint32_t n4 = s_n4, n3 = s_n3;
-            const uint32_t bits2 = NB2 == 16 ? (uint32_t)((const uint16_t*)s_m2)[tid] : ((const uint32_t*)s_m2)[tid];
-            const uint32_t cnt2 = __popc(bits2);
-            const uint32_t inc = warp_incl_scan(cnt2, lane);
-            if (lane == 31) s_scan[warp] = inc;
-            __syncthreads();
-            uint32_t base = 0, n2 = 0;
-#pragma unroll
-            for (int w = 0; w < NW; ++w) {
-                const uint32_t v = s_scan[w];
-                if (w < warp) base += v;
-                n2 += v;
+            uint32_t bits, base;
+            if (NB2 == 16) {
+                const int L = tid >> 2;                          // lane holding M2 bytes 2t, 2t+1
+                const uint32_t wlo = __shfl_sync(PFPL_FULL, m2lo, L & 31);
+                const uint32_t whi = __shfl_sync(PFPL_FULL, m2hi, L & 31);
+                const uint32_t e2 = __shfl_sync(PFPL_FULL, inc2 - pc2, L & 31);
+                const int f = tid & 3;                           // 16-bit field within the lane
+                const uint32_t wsel = f < 2 ? wlo : whi;
+                bits = (wsel >> (16 * (f & 1))) & 0xFFFFu;
+                const uint32_t below = (f >= 2 ? __popc(wlo) : 0u) +
+                                       __popc(wsel & ((f & 1) ? 0xFFFFu : 0u));
+                base = e2 + below;
+            } else {
+                const int L = tid >> 1;                          // lane holding M2 bytes 4t..4t+3
+                const uint32_t wlo = __shfl_sync(PFPL_FULL, m2lo, L & 31);
+                const uint32_t whi = __shfl_sync(PFPL_FULL, m2hi, L & 31);
+                const uint32_t e2 = __shfl_sync(PFPL_FULL, inc2 - pc2, L & 31);
+                bits = (tid & 1) ? whi : wlo;
+                base = e2 + ((tid & 1) ? __popc(wlo) : 0u);
             }
-            base += inc - cnt2;
-            const uint8_t* z2 = pay + 4 + n4 + n3;
-            uint32_t wv[NWD2];
-            uint32_t anyseg = 0;
+            uint32_t wv[NB2 / 4];
+            if (bits == 0) {
+                const uint32_t b = base ? z2[base - 1] : 0u;
 #pragma unroll
-            for (int i = 0; i < NWD2; ++i) {
-                uint32_t w = 0;
+                for (int i = 0; i < NB2 / 4; ++i) wv[i] = b * 0x01010101u;
+            } else {
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    const int bit = 4 * i + k;
-                    const uint32_t cj = base + __popc(bits2 & (bit == 31 ? 0xFFFFFFFFu : ((2u << bit) - 1u)));
-                    w |= (cj ? (uint32_t)z2[cj - 1] : 0u) << (8 * k);
-                }
-                wv[i] = w;
-                if (w) anyseg |= 1u << (i / 4);
-            }
+                for (int i = 0; i < NB2 / 4; ++i) {
+                    uint32_t w = 0;
 #pragma unroll
-            for (int i = 0; i < NWD2; i += 4)
-                *(uint4*)(s_m1 + NB2 * tid + 4 * i) = make_uint4(wv[i], wv[i + 1], wv[i + 2], wv[i + 3]);
-            // 16-byte segment g of M1 = (plane g / NW, warp g % NW)
-#pragma unroll
-            for (int sgi = 0; sgi < NB2 / 16; ++sgi) {
-                if (anyseg & (1u << sgi)) {
-                    const int g = (NB2 / 16) * tid + sgi;
-                    atomicOr(&s_act[g % NW], (ActT)1 << (g / NW));
+                    for (int k = 0; k < 4; ++k) {
+                        const int bit = 4 * i + k;
+                        const uint32_t cj = base + __popc(bits & (bit == 31 ? 0xFFFFFFFFu : ((2u << bit) - 1u)));
+                        w |= (cj ? (uint32_t)z2[cj - 1] : 0u) << (8 * k);
+                    }
+                    wv[i] = w;
                 }
             }
-            if (tid == 0 && 4 + n4 + n3 + n2 > size) s_bad = 1;
-            if (tid == 0) s_n1 = 4 + n4 + n3 + n2;   // temporarily: offset of Z1 in the payload
+#pragma unroll
+            for (int i = 0; i < NB2 / 4; i += 4)
+                *(uint4*)(S.m1 + NB2 * tid + 4 * i) = make_uint4(wv[i], wv[i + 1], wv[i + 2], wv[i + 3]);
+            // 16-byte M1 segment g = (plane g / NWC, warp g % NWC) is non-zero?
+#pragma unroll
+            for (int sg = 0; sg < NB2 / 16; ++sg)
+                S.act[(NB2 / 16) * tid + sg] = (wv[4 * sg] | wv[4 * sg + 1] | wv[4 * sg + 2] | wv[4 * sg + 3]) != 0;
         }
-        __syncthreads();
-        if (s_bad) {
-            if (tid == 0) set_err(p.err);
-            continue;
-        }
+        named_sync(1, NTC);    // M1 and segment flags complete
 
-        // ---- level 1 + inverse bit shuffle ----
-        const uint32_t z1off = s_n1;
-        const uint8_t* z1 = pay + z1off;
-        ActT act = 0;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) act |= s_act[w];
-        // plane p active <=> bit p of act; active low bits P = B - (lowest active plane)
-        const int P = act ? B - (B == 32 ? __ffs((uint32_t)act) - 1 : __ffsll((long long)act) - 1) : 0;
-        uint32_t lo[32], hi[32];
-        if (P == 0) {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) { lo[i] = 0; hi[i] = 0; }
-            if (tid == 0) s_n1 = 0;
-        } else if (B == 32 || P <= 32) {
-            if (P <= 4) rze1_dec<T, 4, 0>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 8) rze1_dec<T, 8, 0>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 16) rze1_dec<T, 16, 0>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else rze1_dec<T, 32, 0>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-        } else {
-            if (P <= 36) rze1_dec<T, 32, 4>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 40) rze1_dec<T, 32, 8>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else if (P <= 48) rze1_dec<T, 32, 16>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
-            else rze1_dec<T, 32, 32>(lo, hi, z1, s_m1, s_wcnt, s_off, &s_n1, tid, lane, warp);
+        // ---- level 1: active planes of this warp, counts, offsets, gather ----
+        int P;
+        {
+            const uint32_t a0 = S.act[lane * NWC + warp];                 // plane p = lane
+            const uint32_t a1 = B == 64 ? S.act[(lane + 32) * NWC + warp] : 0u;
+            const uint32_t ml = __ballot_sync(PFPL_FULL, a0 != 0);        // bit p: plane p
+            const uint32_t mh = __ballot_sync(PFPL_FULL, a1 != 0);        // bit p: plane 32+p
+            // bit b of `all` = bit b of the residuals active (plane B-1-b)
+            const uint64_t all = B == 32 ? (uint64_t)__brev(ml)
+                                         : (((uint64_t)__brev(ml) << 32) | __brev(mh));
+            P = all ? 64 - __clzll((long long)all) : 0;
         }
-        // ---- residual decode + delta decoder's inclusive scan (P:162) ----
+        uint32_t nb[64], ex[16];
+        PFPL_DEC_TIER(dec1_count, S.m1, S, tid, lane, warp, nb, ex);
+        named_sync(1, NTC);    // counts visible
+        uint32_t offl, offh, n1;
+        {
+            uint32_t myl = 0, myh = 0, tl = 0, th = 0;
+#pragma unroll
+            for (int w = 0; w < NWC; ++w) {
+                const uint32_t a = S.wcnt[w][lane];
+                const uint32_t b = B == 64 ? S.wcnt[w][32 + lane] : 0u;
+                if (w < warp) { myl += a; myh += b; }
+                tl += a;
+                th += b;
+            }
+            uint32_t sl = tl, sh = th;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t a = __shfl_down_sync(PFPL_FULL, sl, d);
+                const uint32_t b = B == 64 ? __shfl_down_sync(PFPL_FULL, sh, d) : 0u;
+                if (lane + d < 32) { sl += a; sh += b; }
+            }
+            const uint32_t tot_h = B == 64 ? __shfl_sync(PFPL_FULL, sh, 0) : 0u;
+            const uint32_t tot_l = __shfl_sync(PFPL_FULL, sl, 0);
+            offl = tot_h + sl - tl + myl;
+            offh = sh - th + myh;
+            n1 = tot_l + tot_h;
+        }
+        const uint8_t* z1 = z2 + n2;
+        const bool consistent = 4 + n4 + n3 + n2 + n1 == md.size;
+        uint32_t lo[32], hi[32];
+        PFPL_DEC_TIER(dec1_gather, lo, hi, z1, lane, nb, ex, offl, offh);
+
+        // ---- residual decode + delta decoder's inclusive scan (P:125, P:162) ----
         W dq[32];
         W tsum = 0;
 #pragma unroll
@@ -331,43 +400,45 @@ __global__ void __launch_bounds__(Tr<T>::NT) decode_kernel(const DecParams p) {
             const W t = __shfl_up_sync(PFPL_FULL, incw, d);
             if (lane >= d) incw += t;
         }
-        if (lane == 31) s_scanw[warp] = incw;
-        __syncthreads();   // all Z1 reads done; totals visible
+        if (lane == 31) S.wtot[warp] = (unsigned long long)incw;
+        if (tid == 0) bulk_wait_read0();     // previous chunk's TMA store has read the staging
+        named_sync(1, NTC);    // payload of stage s consumed; warp totals visible
+        if (tid == 0) mbar_arrive(smem_u32(&S.empty[s]));
+        if (!__all_sync(PFPL_FULL, consistent) && lane == 0) set_err(p.err);
         W carry = incw - tsum;
 #pragma unroll
-        for (int w = 0; w < NW; ++w)
-            if (w < warp) carry += s_scanw[w];
-        if (tid == 0 && z1off + s_n1 != size) s_bad = 1;
-        // ---- dequantize into padded rows ----
-        {
-            uint4* row = (uint4*)(s_buf + tid * ROWB);
-#pragma unroll
-            for (int j = 0; j < 2 * S; ++j) {
-                T x[16 / S];
-#pragma unroll
-                for (int i = 0; i < 16 / S; ++i) x[i] = dequantize<T, MODE>(q, (W)(carry + dq[j * (16 / S) + i]), raw);
-                uint4 v;
-                memcpy(&v, x, 16);
-                row[j] = v;
-            }
-        }
-        __syncthreads();
-        if (s_bad) {
-            if (tid == 0) set_err(p.err);
-            continue;
-        }
+        for (int w = 0; w < NWC; ++w)
+            if (w < warp) carry += (W)S.wtot[w];
+
+        // ---- dequantize into swizzled rows ----
         if (m == CW) {
 #pragma unroll
-            for (int i = 0; i < 1024 / NT; ++i) {
-                const int k = i * NT + tid;
-                const uint4 v = *(const uint4*)(s_buf + (k / (2 * S)) * ROWB + (k % (2 * S)) * 16);
-                *(uint4*)(dstc + 16 * k) = v;
+            for (int i = 0; i < 2 * S_; ++i) {
+                T x[16 / S_];
+#pragma unroll
+                for (int k = 0; k < 16 / S_; ++k)
+                    x[k] = dequantize<T, MODE>(q, (W)(carry + dq[i * (16 / S_) + k]), raw);
+                uint4 v;
+                memcpy(&v, x, 16);
+                const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                *(uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4)) = v;
+            }
+            fence_proxy_async();
+            named_sync(1, NTC);    // staging complete
+            if (tid == 0) {
+                tma_store_2d(&tmap, 0, (int)(c * 128), smem_u32(stage_out));
+                bulk_commit();
             }
         } else {
-            for (uint32_t e = tid; e < m; e += NT)
-                ((T*)dstc)[e] = *(const T*)(s_buf + (e / 32) * ROWB + (e % 32) * S);
+            // tail chunk: plain stores of the first m values
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+                const uint32_t e = 32 * tid + i;
+                if (e < m) ((T*)dstc)[e] = dequantize<T, MODE>(q, (W)(carry + dq[i]), raw);
+            }
         }
     }
+    if (tid == 0) bulk_wait0();    // all TMA stores of this CTA complete before exit
 }
 
 template <typename T, int MODE, bool MSR>
@@ -384,6 +455,8 @@ static void* pick_dec(int dtype, int mode, bool ms) {
 #undef PFPL_D
 }
 
+static int dec_threads(int dtype) { return (dtype == 0 ? Tr<float>::NT : Tr<double>::NT) + 32; }
+
 int decode_grid(int dtype, int mode, bool ms, uint64_t C) {
     static int cache[2][4][2] = {};
     int& g = cache[dtype][mode][ms];
@@ -391,18 +464,32 @@ int decode_grid(int dtype, int mode, bool ms, uint64_t C) {
         int dev = 0, sms = 148, per = 1;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        const int nt = dtype == 0 ? Tr<float>::NT : Tr<double>::NT;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, pick_dec(dtype, mode, ms), nt, 0);
+        void* fn = pick_dec(dtype, mode, ms);
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, DEC_SMEM);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, dec_threads(dtype), DEC_SMEM);
         g = sms * (per > 0 ? per : 1);
     }
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
 }
 
+int decode_tickets_per_cta() { return 2; }
+
+cudaError_t make_row_tmap(const void* base, uint64_t bytes, CUtensorMap* map);
+
 cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
                           cudaStream_t s) {
-    const int nt = dtype == 0 ? Tr<float>::NT : Tr<double>::NT;
-    void* args[] = {(void*)&p};
-    return cudaLaunchKernel(pick_dec(dtype, mode, ms), dim3(grid), dim3(nt), args, 0, s);
+    alignas(64) CUtensorMap map;
+    cudaError_t e = make_row_tmap(p.out, p.n * (dtype == 0 ? 4u : 8u), &map);
+    if (e != cudaSuccess) return e;
+    void* fn = pick_dec(dtype, mode, ms);
+    static bool prepared[2][4][2] = {};
+    if (!prepared[dtype][mode][ms]) {
+        e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, DEC_SMEM);
+        if (e != cudaSuccess) return e;
+        prepared[dtype][mode][ms] = true;
+    }
+    void* args[] = {(void*)&p, (void*)&map};
+    return cudaLaunchKernel(fn, dim3(grid), dim3(dec_threads(dtype)), args, DEC_SMEM, s);
 }
 
 }  // namespace pfpl

@@ -80,6 +80,7 @@ cudaError_t launch_header_only(uint8_t* out, uint64_t n, int dtype, int bound, d
 int encode_grid(int dtype, int mode, bool ms, uint64_t C);
 int encode_stages();
 int decode_grid(int dtype, int mode, bool ms, uint64_t C);
+int decode_tickets_per_cta();
 
 // host-side portable log2 (same operation sequence as the device code)
 float log2p_host_f32(float a);
