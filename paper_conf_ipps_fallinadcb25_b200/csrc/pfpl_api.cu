@@ -37,6 +37,8 @@ struct Scratch {
     uint8_t* hdr_host = nullptr;     // pinned 64 bytes
     uint32_t* table_dev = nullptr;   // for pfpl_decompress_chunks
     uint64_t table_cap = 0;
+    uint64_t* offs = nullptr;        // decoder chunk offsets (C + 1)
+    uint64_t offs_cap = 0;
 };
 
 std::mutex g_mu;
@@ -327,8 +329,19 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     Scratch* sc = nullptr;
     st = get_scratch(s, nchunks, &sc);
     if (st != PFPL_OK) return st;
+    if (nchunks + 1 > sc->offs_cap) {
+        if (sc->offs) CK(cudaFreeAsync(sc->offs, s));
+        sc->offs_cap = nchunks + 1 < 1024 ? 1024 : (nchunks + 1) + (nchunks + 1) / 4;
+        CK(cudaMallocAsync(&sc->offs, sc->offs_cap * sizeof(uint64_t), s));
+    }
+    // d1: prefix sum of the stored sizes -> chunk offsets
+    CK(launch_size_scan(table_dev, nchunks, nloc, (uint32_t)cw, (uint32_t)tsz(dtype), payload_bytes,
+                        sc->offs, sc->status, sc->epoch, sc->ticket, sc->ticket_val, err_dev, s));
+    g_launches += 1;
+    sc->ticket_val += (uint64_t)scan_grid(nchunks);
     DecParams p;
     memset(&p, 0, sizeof(p));
+    p.offs = sc->offs;
     p.in = payload;
     p.in_bytes = payload_bytes;
     p.table = table_dev;
@@ -342,6 +355,7 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     p.qc = qc;
     p.err = err_dev;
     p.wd = watchdog_ptr();
+    p.c23 = dtype == PFPL_F32 ? f2u_h(u2f_h((uint32_t)qc.c) * 8388608.0f) : 0u;   // exact or inf
     const bool ms = (flags & HF_MS) != 0;
     const int grid = decode_grid(dtype, mode, ms, nchunks);
     CK(launch_decode(dtype, mode, ms, p, grid, s));
@@ -573,7 +587,7 @@ int pfpl_release_scratch(void) {
         cudaDeviceSynchronize();
         cudaFree(sc->status); cudaFree(sc->ticket); cudaFree(sc->qc_dev); cudaFree(sc->mnmx);
         cudaFree(sc->partial); cudaFree(sc->result); cudaFreeHost(sc->host);
-        cudaFreeHost(sc->hdr_host); cudaFree(sc->table_dev);
+        cudaFreeHost(sc->hdr_host); cudaFree(sc->table_dev); cudaFree(sc->offs);
         delete sc;
         it = g_scratch.erase(it);
     }

@@ -6,12 +6,12 @@
 //
 //   IO warp                                   compute warps (4 for f32, 2 for f64)
 //   -------                                   ------------------------------------
-//   ticket c; chunk offset = prefix of the     wait full[s]; repeat levels 4 -> 2
-//   stored sizes by a look-back over the rebuilt top-down with popcount
-//   size table, which never waits:     prefix ranks -- every warp
-//   all sizes are known; validate; load the    derives M3/M2 itself, no barrier;
-//   payload into stage s with cp.async.bulk    zero level: gather the plane
-//   (2-stage ring)                             words from Z1, inverse bit shuffle in
+//   ticket c; chunk offset from the prefix     wait for chunk k's payload; repeat
+//   sum of the stored sizes (computed   levels 4 -> 2 rebuilt top-down
+//   by size_scan_kernel just before);          with popcount prefix ranks --
+//   validate; load the payload into a byte     every warp derives M3/M2 itself, no
+//   ring with cp.async.bulk, up to 8 chunks    barrier; zero level: gather the
+//   ahead                                      plane words from Z1, inverse shuffle in
 //                                              registers, negabinary^-1 and
 //                                              the delta decoder's inclusive scan
 //                                              (the decode bottleneck P:302),
@@ -23,13 +23,12 @@
 
 namespace pfpl {
 
-constexpr int DIN = 2;                 // payload stages
-constexpr int DSTG = 16448;            // payload stage bytes (16384 + alignment slack)
-constexpr int DOUT_OFF = DIN * DSTG;   // swizzled output staging (1024-aligned below)
+constexpr int NQD = 8;                 // chunks in flight per CTA (payload queue depth)
+constexpr int RING = 32768;            // circular payload ring (bytes, multiple of 16)
 
-struct DecMeta {
+struct DecEntry {
     unsigned long long c;
-    uint32_t size, delta, bad, pad;
+    uint32_t pos, size, delta, bad, rend, pad;
 };
 
 struct DecShared {
@@ -37,11 +36,13 @@ struct DecShared {
     uint8_t act[128];                  // non-zero flag per 16-byte M1 segment
     uint8_t wcnt[4][64];
     unsigned long long wtot[4];        // per-warp totals of the delta scan
-    DecMeta meta[DIN];
-    unsigned long long full[DIN], empty[DIN];
+    DecEntry q[NQD];
+    unsigned long long full[NQD], empty[NQD];
+    uint32_t tail;                     // ring bytes released by the compute warps (monotone)
 };
-constexpr int DOUT = (DOUT_OFF + 1023) & ~1023;
-constexpr int DSH_OFF = DOUT + 16384;
+constexpr int DOUT = 0;                // swizzled output staging (1024-aligned)
+constexpr int DRING = 16384;
+constexpr int DSH_OFF = DRING + RING + 64;
 constexpr int DEC_SMEM = DSH_OFF + (int)sizeof(DecShared);
 static_assert(DEC_SMEM <= 57344, "4 CTAs per SM need <= 56 KiB of shared memory each");
 
@@ -101,6 +102,10 @@ __device__ __forceinline__ void dec1_gather(uint32_t (&lo)[32], uint32_t (&hi)[3
                            __byte_perm(ex[j / 4], 0, 0x4440 + (j % 4));
         const uint32_t n = nb[j];
         uint32_t w = 0, r = o;
+        if (!__any_sync(PFPL_FULL, n != 0)) {              // plane empty in this warp
+            if (j < KL) lo[j] = 0; else hi[j - KL] = 0;
+            continue;
+        }
         if (n & 1u) w |= (uint32_t)z1[r++];
         if (n & 2u) w |= (uint32_t)z1[r++] << 8;
         if (n & 4u) w |= (uint32_t)z1[r++] << 16;
@@ -147,16 +152,18 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     extern __shared__ __align__(1024) uint8_t smem[];
     DecShared& S = *reinterpret_cast<DecShared*>(smem + DSH_OFF);
     uint8_t* const stage_out = smem + DOUT;
+    uint8_t* const ring = smem + DRING;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint64_t C = p.C;
 
     if (tid == 0) {
         g_pfpl_wd = p.wd;
         if (smem_u32(smem) & 1023u) __trap();
-        for (int s = 0; s < DIN; ++s) {
-            mbar_init(smem_u32(&S.full[s]), 1);
-            mbar_init(smem_u32(&S.empty[s]), 1);
+        for (int k = 0; k < NQD; ++k) {
+            mbar_init(smem_u32(&S.full[k]), 1);
+            mbar_init(smem_u32(&S.empty[k]), 1);
         }
+        S.tail = 0;
         fence_barrier_init();
         prefetch_tmap(&tmap);
     }
@@ -164,53 +171,53 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
 
     if (warp == NWC) {
         // =========================== IO warp ===========================
-        const uint64_t EP = (uint64_t)p.epoch << 48;
         unsigned long long tnext = 0;
+        uint32_t head = 0;
         if (lane == 0) tnext = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-        for (uint32_t it = 0;; ++it) {
-            const int s = it % DIN;
+        for (uint32_t k = 0;; ++k) {
+            const int slot = k % NQD;
             const unsigned long long c = __shfl_sync(PFPL_FULL, tnext, 0);
             if (lane == 0) tnext = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-            mbar_wait_wd(smem_u32(&S.empty[s]), ((it / DIN) & 1u) ^ 1u, 0x21);
             if (c >= C) {
+                mbar_wait_wd(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
                 if (lane == 0) {
-                    S.meta[s].c = c;
-                    mbar_arrive(smem_u32(&S.full[s]));
+                    S.q[slot].c = c;
+                    mbar_arrive(smem_u32(&S.full[slot]));
                 }
                 break;
             }
-            // d1: offset = sum of the stored sizes before c (look-back)
+            // d1: chunk offset from the size-table prefix sum (size_scan_kernel)
             const uint32_t size = p.table[c];
-            uint64_t excl = 0;
-            for (int64_t look = (int64_t)c - 1; look >= 0; look -= 32) {
-                const int64_t idx = look - lane;
-                uint64_t val = 0;
-                bool isP = false;
-                if (idx >= 0) {
-                    const uint64_t d = ld_relaxed(&p.status[idx]);
-                    if ((uint32_t)(d >> 48) == p.epoch && ((d >> 46) & 3u) == LB_P) { isP = true; val = d & LB_VAL; }
-                    else val = p.table[idx];
-                }
-                const uint32_t pm = __ballot_sync(PFPL_FULL, isP);
-                if (pm) {
-                    const int first = __ffs(pm) - 1;
-                    excl += warp_sum64(lane <= first ? val : 0ull);
-                    break;
-                }
-                excl += warp_sum64(val);
-            }
+            const uint64_t excl = p.offs[c];
             const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
             const uint32_t rawb = m * S_;
             uint32_t bad = 0;
-            if (size > rawb || excl + size > p.in_bytes) bad = 1;
-            if (c == C - 1 && excl + size != p.in_bytes) bad = 1;
-            if (size < 4 && size != rawb) bad = 1;
-            if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | ((excl + size) & LB_VAL));
-            // stage the payload: 16-byte aligned superset by one bulk copy (never
-            // past the last 16-byte boundary of the stream), the rest by the lanes
-            uint8_t* stg = smem + s * DSTG;
+            if (size > rawb || excl + size > p.in_bytes || (size < 4 && size != rawb)) bad = 1;
+            // reserve a ring slice for the 16-byte aligned superset of the payload
             const uint8_t* g = p.in + excl;
             const uint32_t delta = (uint32_t)((uintptr_t)g & 15u);
+            const uint32_t R = bad ? 16u : ((delta + size + 15u) & ~15u) + 16u;
+            const uint32_t head0 = head;
+            if (head % RING + R > (uint32_t)RING) head += RING - head % RING;   // never wrap a slice
+            // live bytes are [tail, head0): free if empty or span <= RING
+            auto full = [&]() {
+                const uint32_t t = *(volatile uint32_t*)&S.tail;
+                return t != head0 && head + R - t > (uint32_t)RING;
+            };
+            if (full()) {
+                const uint64_t t0 = globaltimer();
+                uint32_t ns = 64;
+                while (full()) {
+                    if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x23, head);
+                    __nanosleep(ns);
+                    ns = ns < 2048 ? 2 * ns : ns;
+                }
+            }
+            const uint32_t pos = head % RING;
+            head += R;
+            mbar_wait_wd(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
+            // bulk copy of the aligned superset, never past the last 16-byte
+            // boundary of the stream; the remainder by the lanes
             const uint8_t* a0 = g - delta;
             const uint8_t* want = g + size;
             const uint8_t* a1 = (const uint8_t*)(((uintptr_t)want + 15u) & ~(uintptr_t)15u);
@@ -218,20 +225,23 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             if (a1 > lim) a1 = lim;
             if (a1 < a0) a1 = a0;
             const uint32_t bulk = bad ? 0u : (uint32_t)(a1 - a0);
+            uint8_t* stg = ring + pos;
             if (!bad)
                 for (const uint8_t* q = a1 + lane; q < want; q += 32) stg[q - a0] = *q;
             __syncwarp();
             if (lane == 0) {
-                DecMeta& md = S.meta[s];
-                md.c = c;
-                md.size = size;
-                md.delta = delta;
-                md.bad = bad;
+                DecEntry& e = S.q[slot];
+                e.c = c;
+                e.pos = pos;
+                e.size = size;
+                e.delta = delta;
+                e.bad = bad;
+                e.rend = head;
                 if (bulk) {
-                    mbar_arrive_tx(smem_u32(&S.full[s]), bulk);
-                    bulk_g2s(smem_u32(stg), a0, bulk, smem_u32(&S.full[s]));
+                    mbar_arrive_tx(smem_u32(&S.full[slot]), bulk);
+                    bulk_g2s(smem_u32(stg), a0, bulk, smem_u32(&S.full[slot]));
                 } else {
-                    mbar_arrive(smem_u32(&S.full[s]));
+                    mbar_arrive(smem_u32(&S.full[slot]));
                 }
             }
         }
@@ -242,18 +252,27 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     QF<T> q;
     q.load(p.qc);
     const bool raw = (p.qc.flags & HF_RAWWORDS) != 0;
+    const float c23 = u2f((uint32_t)p.c23);
+    const bool fastdq = sizeof(T) == 4 && MODE == MODE_ABS && !isinf(c23);
     for (uint32_t it = 0;; ++it) {
-        const int s = it % DIN;
-        mbar_wait_wd(smem_u32(&S.full[s]), (it / DIN) & 1u, 0x22);
-        const DecMeta md = S.meta[s];
+        const int slot = it % NQD;
+        mbar_wait_wd(smem_u32(&S.full[slot]), (it / NQD) & 1u, 0x22);
+        const DecEntry md = S.q[slot];
         const uint64_t c = md.c;
         if (c >= C) break;
         const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
-        const uint8_t* pay = smem + s * DSTG + md.delta;
+        const uint8_t* pay = ring + md.pos + md.delta;
         uint8_t* const dstc = (uint8_t*)p.out + c * (uint64_t)kChunkBytes;
+        auto release = [&]() {
+            if (tid == 0) {
+                *(volatile uint32_t*)&S.tail = md.rend;
+                mbar_arrive(smem_u32(&S.empty[slot]));
+            }
+        };
         if (md.bad) {
             named_sync(1, NTC);
-            if (tid == 0) { set_err(p.err); mbar_arrive(smem_u32(&S.empty[s])); }
+            if (tid == 0) set_err(p.err);
+            release();
             continue;
         }
         if (md.size == m * S_) {
@@ -265,10 +284,9 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 ((uint32_t*)dstc)[j] = __funnelshift_r(sw[0], sw[1], 8u * a);
             }
             named_sync(1, NTC);
-            if (tid == 0) mbar_arrive(smem_u32(&S.empty[s]));
+            release();
             continue;
         }
-
         // ---- levels 4 -> 3 -> 2, derived by every warp (no barrier) ----
         const uint32_t M4 = (uint32_t)pay[0] | ((uint32_t)pay[1] << 8) | ((uint32_t)pay[2] << 16) |
                             ((uint32_t)pay[3] << 24);
@@ -402,8 +420,8 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         }
         if (lane == 31) S.wtot[warp] = (unsigned long long)incw;
         if (tid == 0) bulk_wait_read0();     // previous chunk's TMA store has read the staging
-        named_sync(1, NTC);    // payload of stage s consumed; warp totals visible
-        if (tid == 0) mbar_arrive(smem_u32(&S.empty[s]));
+        named_sync(1, NTC);    // payload consumed; warp totals visible
+        release();
         if (!__all_sync(PFPL_FULL, consistent) && lane == 0) set_err(p.err);
         W carry = incw - tsum;
 #pragma unroll
@@ -417,7 +435,8 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 T x[16 / S_];
 #pragma unroll
                 for (int k = 0; k < 16 / S_; ++k)
-                    x[k] = dequantize<T, MODE>(q, (W)(carry + dq[i * (16 / S_) + k]), raw);
+                    x[k] = fastdq ? (T)q.abs_dq_fast((uint32_t)(carry + dq[i * (16 / S_) + k]), c23)
+                                  : dequantize<T, MODE>(q, (W)(carry + dq[i * (16 / S_) + k]), raw);
                 uint4 v;
                 memcpy(&v, x, 16);
                 const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);

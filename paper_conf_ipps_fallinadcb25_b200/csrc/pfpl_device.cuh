@@ -116,6 +116,14 @@ PFPL_HD double pow2p_f64(double y) {
     return p * u2d((uint64_t)(ki + 1023) << 52);
 }
 
+// predicated select that the compiler cannot turn into a branch
+__device__ __forceinline__ uint32_t selp_u32(uint32_t a, uint32_t b, bool p) {
+    uint32_t r;
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\tselp.b32 %0, %1, %2, q;\n\t}"
+        : "=r"(r) : "r"(a), "r"(b), "r"((uint32_t)p));
+    return r;
+}
+
 // ------------------------------------------------------------------------
 // quantizers: value -> word (bin code or raw bits)
 // ------------------------------------------------------------------------
@@ -167,6 +175,14 @@ template <> struct QF<float> {
     __device__ __forceinline__ float abs_dq(uint32_t w) const {
         return w < 0x00800000u ? __int2float_rn(unzz(w)) * c : u2f(w);
     }
+    // same value without the XU pipe: |b| = (z+1)>>1, bits(2^23 + |b|) = (z + 0x96000001) >> 1,
+    // fl(|b| * eb2) = fma(2^23 + |b|, eb2, -2^23*eb2) (one rounding of the exact product;
+    // c23 = 2^23*eb2 must be finite), sign from the zigzag LSB.
+    __device__ __forceinline__ float abs_dq_fast(uint32_t w, float c23) const {
+        const float f = u2f((w + 0x96000001u) >> 1);
+        const float mag = __fmaf_rn(f, c, -c23);
+        return u2f(selp_u32(f2u(mag) ^ (w * 0x80000000u), w, w < 0x00800000u));
+    }
     // REL: a = c_lo, b = w, c = inv_w.  log-space bin (R5), conservative
     // 1-ulp-shrunk check (R7), sign+bin in the negative-NaN payload (R10),
     // sign and exponent bits of every word inverted (R11).
@@ -215,6 +231,7 @@ template <> struct QF<double> {
         return ok ? zz(bi) : d2u(v);
     }
     __device__ __forceinline__ uint64_t abs_qb(double v) const { return abs_q(v); }
+    __device__ __forceinline__ double abs_dq_fast(uint32_t, float) const { return 0.0; }   // f32 only
     __device__ __forceinline__ double abs_dq(uint64_t w) const {
         return w < 0x0010000000000000ull ? __ll2double_rn((long long)unzz(w)) * c : u2d(w);
     }
@@ -365,8 +382,12 @@ template <int K> __device__ __forceinline__ void transpose_inv(uint32_t (&r)[32]
 #pragma unroll
     for (int w = 0; w < K; ++w) {
 #pragma unroll
-        for (int h = H - 1; h >= 0; --h)
-            r[w + K * h] = K == 32 ? r[w] : ((r[w] >> (K * h)) & ((1u << (K & 31)) - 1u));
+        for (int h = H - 1; h >= 0; --h) {
+            if (K == 32) r[w + K * h] = r[w];
+            else if (K == 8) r[w + K * h] = __byte_perm(r[w], 0, 0x4440 + h);            // 1 PRMT
+            else if (K == 16) r[w + K * h] = __byte_perm(r[w], 0, h ? 0x4432 : 0x4410);
+            else r[w + K * h] = (r[w] >> (K * h)) & ((1u << (K & 31)) - 1u);
+        }
     }
 }
 
@@ -496,12 +517,24 @@ __device__ __forceinline__ bool mbar_try(uint32_t a, uint32_t parity) {
         "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(r) : "r"(a), "r"(parity) : "memory");
     return r != 0;
 }
-__device__ __forceinline__ void mbar_wait_wd(uint32_t a, uint32_t parity, uint32_t site) {
+// try_wait with a suspend-time hint: the thread is parked by the hardware until
+// the phase completes (or the hint expires), so waiting does not spin on the
+// issue port
+__device__ __forceinline__ bool mbar_try_hint(uint32_t a, uint32_t parity, uint32_t ns) {
+    uint32_t r;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(r) : "r"(a), "r"(parity), "r"(ns) : "memory");
+    return r != 0;
+}
+__device__ __forceinline__ void mbar_wait_wd(uint32_t a, uint32_t parity, uint32_t site,
+                                             uint32_t hint_ns = 20000) {
     if (mbar_try(a, parity)) return;
     const uint64_t t0 = globaltimer();
-    for (uint32_t i = 1;; ++i) {
-        if (mbar_try(a, parity)) return;
-        if ((i & 63u) == 0 && globaltimer() - t0 > kWatchdogNs) watchdog_fire(site, parity);
+    for (;;) {
+        if (mbar_try_hint(a, parity, hint_ns)) return;
+        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(site, parity);
     }
 }
 __device__ __forceinline__ void fence_barrier_init() {

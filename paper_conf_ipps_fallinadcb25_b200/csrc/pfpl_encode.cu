@@ -107,12 +107,20 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
 __device__ __forceinline__ uint32_t slice_bytes(uint32_t n1) { return (ZPRE + n1 + 15u) & ~15u; }
 __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
     const uint32_t R = slice_bytes(n1);
-    uint32_t head = S.head;
+    const uint32_t head0 = S.head;
+    uint32_t head = head0;
     const uint32_t p0 = head % ARENA;
     if (p0 + R > (uint32_t)ARENA) head += ARENA - p0;      // a slice never wraps
-    if (lane == 0 && head + R - ld_volatile_u32(&S.tail) > (uint32_t)ARENA) {
+    // live bytes are [tail, head0); the new slice [head, head+R) is free when the
+    // arena is empty or the live range plus the slice spans at most ARENA bytes
+    // (the gap skipped to avoid wrapping is never released by itself)
+    auto full = [&]() {
+        const uint32_t t = ld_volatile_u32(&S.tail);
+        return t != head0 && head + R - t > (uint32_t)ARENA;
+    };
+    if (lane == 0 && full()) {
         const uint64_t t0 = globaltimer();
-        while (head + R - ld_volatile_u32(&S.tail) > (uint32_t)ARENA) {
+        while (full()) {
             if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x13, head);
             __nanosleep(64);
         }

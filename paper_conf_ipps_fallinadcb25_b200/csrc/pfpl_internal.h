@@ -60,6 +60,8 @@ struct DecParams {
     uint32_t epoch;
     QConst qc;               // a/b/c as in QConst; decoder uses eb2 (ABS/NOA) or w (REL)
     int* err;                // set to PFPL_ERR_CORRUPT on malformed chunks
+    uint64_t c23;            // f32 ABS: bits of 2^23 * eb2 (inf if it overflows)
+    const uint64_t* offs;    // offs[c] = byte offset of chunk c's payload (size_scan_kernel)
     unsigned int* wd;        // watchdog report (mapped host memory) or null
 };
 
@@ -68,6 +70,12 @@ cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int 
                           cudaStream_t s);
 cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
                           cudaStream_t s);
+int scan_grid(uint64_t C);
+cudaError_t launch_size_scan(const uint32_t* table, uint64_t C, uint64_t n, uint32_t cw,
+                             uint32_t s_bytes, uint64_t in_bytes, uint64_t* offs,
+                             unsigned long long* status, uint32_t epoch,
+                             unsigned long long* ticket, uint64_t tbase, int* err,
+                             cudaStream_t s);
 cudaError_t launch_minmax(int dtype, const void* in, uint64_t n, double* partial,
                           int blocks, cudaStream_t s);
 cudaError_t launch_minmax_final(const double* partial, int blocks, double* mnmx,

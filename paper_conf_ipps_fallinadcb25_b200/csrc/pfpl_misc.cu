@@ -125,6 +125,106 @@ __global__ void header_only_kernel(uint8_t* out, uint64_t n, int dtype, int boun
     result[0] = 48;
 }
 
+// ---------------------------------------------------------------------------
+// d1: exclusive prefix sum of the stored chunk sizes ("the decoder
+// computes a prefix sum over the stored chunk sizes"), one pass with a
+// decoupled look-back over 8192-entry tiles.  offs[c] = byte offset of chunk c
+// in the payload area; offs[C] = total.  Sizes are validated against the raw
+// chunk size; the total must equal the payload bytes (else *err = CORRUPT).
+// ---------------------------------------------------------------------------
+constexpr int SCAN_T = 256, SCAN_PER = 32, SCAN_TILE = SCAN_T * SCAN_PER;
+
+__global__ void __launch_bounds__(SCAN_T) size_scan_kernel(const uint32_t* table, uint64_t C,
+                                                            uint64_t n, uint32_t cw, uint32_t s_bytes,
+                                                            uint64_t in_bytes, uint64_t* offs,
+                                                            unsigned long long* status, uint32_t epoch,
+                                                            unsigned long long* ticket, uint64_t tbase,
+                                                            int* err) {
+    __shared__ unsigned long long sh_tile;
+    __shared__ uint64_t wsum[SCAN_T / 32];
+    __shared__ uint64_t sh_excl;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) sh_tile = atomicAdd(ticket, 1ull) - tbase;
+    __syncthreads();
+    const uint64_t t = sh_tile;
+    const uint64_t c0 = t * SCAN_TILE + (uint64_t)tid * SCAN_PER;
+    uint64_t v[SCAN_PER];
+    uint64_t sum = 0;
+    bool bad = false;
+#pragma unroll
+    for (int i = 0; i < SCAN_PER; ++i) {
+        const uint64_t c = c0 + i;
+        uint64_t sz = 0;
+        if (c < C) {
+            sz = table[c];
+            const uint64_t m = c + 1 < C ? cw : n - c * cw;
+            if (sz > m * s_bytes || (sz < 4 && sz != m * s_bytes)) bad = true;
+        }
+        v[i] = sum;
+        sum += sz;
+    }
+    uint64_t inc = warp_incl_scan64(sum, lane);
+    if (lane == 31) wsum[warp] = inc;
+    __syncthreads();
+    uint64_t before = 0, agg = 0;
+#pragma unroll
+    for (int w = 0; w < SCAN_T / 32; ++w) {
+        if (w < warp) before += wsum[w];
+        agg += wsum[w];
+    }
+    if (warp == 0) {
+        const uint64_t EP = (uint64_t)epoch << 48;
+        if (lane == 0) st_relaxed(&status[t], EP | ((t == 0 ? LB_P : LB_A) << 46) | agg);
+        uint64_t excl = 0;
+        if (t > 0) {
+            int64_t look = (int64_t)t - 1;
+            for (;;) {
+                const int64_t idx = look - lane;
+                uint64_t val = 0, flag = LB_P;
+                if (idx >= 0) {
+                    for (;;) {
+                        const uint64_t d = ld_relaxed(&status[idx]);
+                        flag = ((uint32_t)(d >> 48) == epoch) ? ((d >> 46) & 3u) : 0u;
+                        if (flag) { val = d & LB_VAL; break; }
+                    }
+                }
+                const uint32_t pm = __ballot_sync(PFPL_FULL, flag == LB_P);
+                if (pm) {
+                    const int first = __ffs(pm) - 1;
+                    excl += warp_sum64(lane <= first ? val : 0ull);
+                    break;
+                }
+                excl += warp_sum64(val);
+                look -= 32;
+            }
+            if (lane == 0) st_relaxed(&status[t], EP | (LB_P << 46) | (excl + agg));
+        }
+        if (lane == 0) sh_excl = excl;
+    }
+    __syncthreads();
+    const uint64_t base = sh_excl + before + inc - sum;
+#pragma unroll
+    for (int i = 0; i < SCAN_PER; ++i) {
+        const uint64_t c = c0 + i;
+        if (c < C) offs[c] = base + v[i];
+        if (c == C - 1 && base + v[i] + table[c] != in_bytes) bad = true;
+        if (c == C - 1) offs[C] = base + v[i] + table[c];
+    }
+    if (bad) atomicExch(err, -4);
+}
+
+int scan_grid(uint64_t C) { return (int)((C + SCAN_TILE - 1) / SCAN_TILE); }
+
+cudaError_t launch_size_scan(const uint32_t* table, uint64_t C, uint64_t n, uint32_t cw,
+                             uint32_t s_bytes, uint64_t in_bytes, uint64_t* offs,
+                             unsigned long long* status, uint32_t epoch,
+                             unsigned long long* ticket, uint64_t tbase, int* err,
+                             cudaStream_t s) {
+    size_scan_kernel<<<scan_grid(C), SCAN_T, 0, s>>>(table, C, n, cw, s_bytes, in_bytes, offs,
+                                                     status, epoch, ticket, tbase, err);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_minmax(int dtype, const void* in, uint64_t n, double* partial, int blocks,
                           cudaStream_t s) {
     if (dtype == 0) minmax_kernel<float><<<blocks, MM_THREADS, 0, s>>>((const float*)in, n, partial);

@@ -3,7 +3,7 @@ import csv, io, subprocess, sys
 from collections import defaultdict, Counter
 rep = sys.argv[1]; per = float(sys.argv[2]) if len(sys.argv) > 2 else 1.0
 top = int(sys.argv[3]) if len(sys.argv) > 3 else 40
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"] + (["--kernel-name", "regex:" + sys.argv[4]] if len(sys.argv) > 4 else []),
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
 cur = None; line = None; agg = defaultdict(Counter); src = {}
