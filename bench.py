@@ -212,10 +212,18 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # PFPL_BENCH_SHARE_GPU=1 maps all ranks onto the visible GPUs round-robin
+    # (functional test of the multi-rank path on a 1-GPU box, with gloo)
+    if os.environ.get("PFPL_BENCH_SHARE_GPU"):
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("PFPL_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     from paper_conf_ipps_fallinadcb25_b200 import _build
     if rank == 0:
         _build.build()
