@@ -14,7 +14,10 @@ import subprocess
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 LIB = os.path.join(PKG, "libpfpl.so")
-SRCS = sorted(glob.glob(os.path.join(PKG, "csrc", "*.cu")))
+SRCS = sorted(f for f in glob.glob(os.path.join(PKG, "csrc", "*.cu")) if not f.endswith("pfpl_inst.cu"))
+INST = os.path.join(PKG, "csrc", "pfpl_inst.cu")
+# (kind, dtype, mode): encoder f32/f64 x ABS/REL/RAW/NOA, decoder f32/f64 x ABS/REL/RAW
+INST_JOBS = [(0, d, m) for d in (0, 1) for m in range(4)] + [(1, d, m) for d in (0, 1) for m in range(3)]
 DEPS = SRCS + glob.glob(os.path.join(PKG, "csrc", "*.h")) + glob.glob(os.path.join(PKG, "csrc", "*.cuh")) \
     + [os.path.join(ROOT, "include", "pfpl.h")]
 
@@ -42,22 +45,30 @@ def needs_build() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS)
 
 
-def build(force: bool = False, verbose: bool = False, jobs: int = 8) -> str:
+def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count() or 8) -> str:
     if not force and not needs_build():
         return LIB
     bdir = os.path.join(ROOT, "build")
     os.makedirs(bdir, exist_ok=True)
-    objs = []
-    procs = []
+    jobs_ = []
     for src in SRCS:
-        obj = os.path.join(bdir, os.path.basename(src) + ".o")
-        objs.append(obj)
-        cmd = [nvcc(), *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-dc" if False else "-c",
-               src, "-o", obj]
-        log = open(obj + ".log", "w")
-        procs.append((subprocess.Popen(cmd, stdout=log, stderr=subprocess.STDOUT), cmd, obj))
-    for p, cmd, obj in procs:
+        jobs_.append((src, os.path.join(bdir, os.path.basename(src) + ".o"), []))
+    for k, d, m in INST_JOBS:
+        jobs_.append((INST, os.path.join(bdir, f"{'enc' if k == 0 else 'dec'}_{d}_{m}.o"),
+                      [f"-DPFPL_KIND={k}", f"-DPFPL_DT={d}", f"-DPFPL_MODE={m}"]))
+    jobs_.sort(key=lambda j: 0 if j[2] else 1)      # long instantiation TUs first
+    objs = [j[1] for j in jobs_]
+    running, pending = [], list(jobs_)
+    while pending or running:
+        while pending and len(running) < max(1, jobs):
+            src, obj, defs = pending.pop(0)
+            cmd = [nvcc(), *NVCC_FLAGS, *defs, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
+            log = open(obj + ".log", "w")
+            running.append((subprocess.Popen(cmd, stdout=log, stderr=subprocess.STDOUT), cmd, obj))
+        p, cmd, obj = running.pop(0)
         if p.wait() != 0:
+            for q, _, _ in running:
+                q.kill()
             raise RuntimeError("nvcc failed: " + " ".join(cmd) + "\n" + open(obj + ".log").read())
         if verbose:
             print(open(obj + ".log").read())

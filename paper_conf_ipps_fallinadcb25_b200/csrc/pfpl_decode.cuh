@@ -18,6 +18,7 @@
 //                                              dequantize into swizzled
 //                                              rows; one thread stores the chunk with
 //                                              a TMA 2-D tensor store
+#pragma once
 #include <cuda.h>
 #include "pfpl_device.cuh"
 
@@ -458,57 +459,6 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         }
     }
     if (tid == 0) bulk_wait0();    // all TMA stores of this CTA complete before exit
-}
-
-template <typename T, int MODE, bool MSR>
-static void* dec_fn() { return (void*)decode_kernel<T, MODE, MSR>; }
-
-static void* pick_dec(int dtype, int mode, bool ms) {
-#define PFPL_D(T)                                                                  \
-    switch (mode) {                                                                \
-        case MODE_ABS: return ms ? dec_fn<T, MODE_ABS, true>() : dec_fn<T, MODE_ABS, false>(); \
-        case MODE_REL: return ms ? dec_fn<T, MODE_REL, true>() : dec_fn<T, MODE_REL, false>(); \
-        default: return ms ? dec_fn<T, MODE_RAW, true>() : dec_fn<T, MODE_RAW, false>();       \
-    }
-    if (dtype == 0) { PFPL_D(float) } else { PFPL_D(double) }
-#undef PFPL_D
-}
-
-static int dec_threads(int dtype) { return (dtype == 0 ? Tr<float>::NT : Tr<double>::NT) + 32; }
-
-int decode_grid(int dtype, int mode, bool ms, uint64_t C) {
-    static int cache[2][4][2] = {};
-    int& g = cache[dtype][mode][ms];
-    if (!g) {
-        int dev = 0, sms = 148, per = 1;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        void* fn = pick_dec(dtype, mode, ms);
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, DEC_SMEM);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, dec_threads(dtype), DEC_SMEM);
-        g = sms * (per > 0 ? per : 1);
-    }
-    return (int)(C < (uint64_t)g ? C : (uint64_t)g);
-}
-
-int decode_tickets_per_cta() { return 2; }
-
-cudaError_t make_row_tmap(const void* base, uint64_t bytes, CUtensorMap* map);
-
-cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
-                          cudaStream_t s) {
-    alignas(64) CUtensorMap map;
-    cudaError_t e = make_row_tmap(p.out, p.n * (dtype == 0 ? 4u : 8u), &map);
-    if (e != cudaSuccess) return e;
-    void* fn = pick_dec(dtype, mode, ms);
-    static bool prepared[2][4][2] = {};
-    if (!prepared[dtype][mode][ms]) {
-        e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, DEC_SMEM);
-        if (e != cudaSuccess) return e;
-        prepared[dtype][mode][ms] = true;
-    }
-    void* args[] = {(void*)&p, (void*)&map};
-    return cudaLaunchKernel(fn, dim3(grid), dim3(dec_threads(dtype)), args, DEC_SMEM, s);
 }
 
 }  // namespace pfpl

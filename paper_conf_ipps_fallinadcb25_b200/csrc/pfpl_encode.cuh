@@ -24,6 +24,7 @@
 // each bit plane are one aligned word of the shuffled chunk.
 // Arena slice of a chunk: [pos, pos + ZPRE + n1) with Z1 at pos + ZPRE and
 // M4 | Z4 | Z3 | Z2 packed immediately before it (section order of R16).
+#pragma once
 #include <cuda.h>
 #include "pfpl_device.cuh"
 
@@ -62,7 +63,7 @@ __device__ __forceinline__ void put_u64(uint8_t* p, uint64_t v) {
     for (int i = 0; i < 8; ++i) p[i] = (uint8_t)(v >> (8 * i));
 }
 
-__device__ void write_header(uint8_t* out, const EncParams& p, const QConst& qc) {
+static __device__ void write_header(uint8_t* out, const EncParams& p, const QConst& qc) {
     out[0] = 'P'; out[1] = 'F'; out[2] = 'P'; out[3] = 'L';
     out[4] = 1; out[5] = (uint8_t)p.dtype; out[6] = (uint8_t)p.bound; out[7] = (uint8_t)qc.flags;
     put_u64(out + 8, p.n_total);
@@ -565,97 +566,6 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         S.q[slot].c = ~0ull;
         mbar_arrive(smem_u32(&S.mq_full[slot]));
     }
-}
-
-// ---------------------------------------------------------------------------
-// host side
-// ---------------------------------------------------------------------------
-template <typename T, int MODE, bool MSR>
-static void* enc_fn() { return (void*)encode_kernel<T, MODE, MSR>; }
-
-static void* pick_enc(int dtype, int mode, bool ms) {
-#define PFPL_E(T)                                                                  \
-    switch (mode) {                                                                \
-        case MODE_ABS: return ms ? enc_fn<T, MODE_ABS, true>() : enc_fn<T, MODE_ABS, false>(); \
-        case MODE_REL: return ms ? enc_fn<T, MODE_REL, true>() : enc_fn<T, MODE_REL, false>(); \
-        case MODE_RAW: return ms ? enc_fn<T, MODE_RAW, true>() : enc_fn<T, MODE_RAW, false>(); \
-        default: return ms ? enc_fn<T, MODE_NOA, true>() : enc_fn<T, MODE_NOA, false>();       \
-    }
-    if (dtype == 0) { PFPL_E(float) } else { PFPL_E(double) }
-#undef PFPL_E
-}
-
-static int enc_threads(int dtype) { return (dtype == 0 ? Tr<float>::NT : Tr<double>::NT) + 32; }
-
-static cudaError_t prepare_enc(void* fn) {
-    return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ENC_SMEM);
-}
-
-int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
-    static int cache[2][4][2] = {};
-    int& g = cache[dtype][mode][ms];
-    if (!g) {
-        int dev = 0, sms = 148, per = 1;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        void* fn = pick_enc(dtype, mode, ms);
-        prepare_enc(fn);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, enc_threads(dtype), ENC_SMEM);
-        g = sms * (per > 0 ? per : 1);
-    }
-    return (int)(C < (uint64_t)g ? C : (uint64_t)g);
-}
-
-int encode_stages() { return NIN; }
-
-typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
-                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
-                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
-                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-static EncodeTiledFn get_encode_tiled() {
-    static EncodeTiledFn fn = nullptr;
-    if (!fn) {
-        void* f = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
-            q == cudaDriverEntryPointSuccess)
-            fn = (EncodeTiledFn)f;
-    }
-    return fn;
-}
-
-// 2-D view of the input as 128-byte rows of 32 u32 words; a chunk = 128 rows.
-cudaError_t make_row_tmap(const void* base, uint64_t bytes, CUtensorMap* map) {
-    memset(map, 0, sizeof(*map));
-    const uint64_t rows = bytes / 128;
-    if (rows < 128) return cudaSuccess;            // no full chunk: map never used
-    EncodeTiledFn fn = get_encode_tiled();
-    if (!fn) return cudaErrorNotSupported;
-    cuuint64_t dims[2] = {32, rows};
-    cuuint64_t strides[1] = {128};
-    cuuint32_t box[2] = {32, 128};
-    cuuint32_t es[2] = {1, 1};
-    CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void*>(base), dims, strides,
-                    box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
-}
-
-cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int grid,
-                          cudaStream_t s) {
-    alignas(64) CUtensorMap map;
-    cudaError_t e = make_row_tmap(p.in, p.n * (dtype == 0 ? 4u : 8u), &map);
-    if (e != cudaSuccess) return e;
-    void* fn = pick_enc(dtype, mode, ms);
-    static bool prepared[2][4][2] = {};
-    if (!prepared[dtype][mode][ms]) {
-        e = prepare_enc(fn);
-        if (e != cudaSuccess) return e;
-        prepared[dtype][mode][ms] = true;
-    }
-    void* args[] = {(void*)&p, (void*)&map};
-    return cudaLaunchKernel(fn, dim3(grid), dim3(enc_threads(dtype)), args, ENC_SMEM, s);
 }
 
 }  // namespace pfpl

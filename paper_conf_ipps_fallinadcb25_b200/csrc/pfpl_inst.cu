@@ -1,0 +1,26 @@
+// pfpl_inst.cu -- explicit instantiation of one (dtype, mode) pair of the fused
+// encoder or decoder, so the 28 kernel variants compile in parallel.  Built by
+// _build.py with -DPFPL_KIND=0 (encode) / 1 (decode), -DPFPL_DT, -DPFPL_MODE.
+#if PFPL_KIND == 0
+#include "pfpl_encode.cuh"
+#define PFPL_KERNEL encode_kernel
+#define PFPL_PREFIX enc_ptr_
+#else
+#include "pfpl_decode.cuh"
+#define PFPL_KERNEL decode_kernel
+#define PFPL_PREFIX dec_ptr_
+#endif
+
+#define PFPL_CAT3(a, b, c, d) a##b##_##d
+#define PFPL_NAME(p, d, m) PFPL_CAT3(p, d, _, m)
+
+namespace pfpl {
+#if PFPL_DT == 0
+typedef float InstT;
+#else
+typedef double InstT;
+#endif
+void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms) {
+    return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false>;
+}
+}  // namespace pfpl
