@@ -39,7 +39,7 @@ PAPER_CONTEXT = {"paper_pfpl_cuda_rtx4090_gbs": 423, "paper_pfpl_omp_ryzen2950x_
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="nyx")
@@ -59,62 +59,65 @@ def _peaks():
 
 
 class Clocks:
-    """Sample nvidia-smi clocks/throttle reasons during the timed region."""
+    """Sample SM clocks and clock-event (throttle) reasons DURING the timed region.
 
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap,utilization.gpu")
+    NVML (nvidia-ml-py) polled from a thread every ~0.5 ms: the timed region
+    of a default run is tens of ms, far below nvidia-smi's sampling period.
+    Samples are kept only while `active` is set (the timed loop)."""
+
+    BITS = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20,
+            "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
 
     def __init__(self, index: int):
         self.index = index
-        self.proc = None
-        self.lines = []
+        self.samples = []
+        self.active = False
+        self.stop = False
+        self.err = None
+        self.max_mhz = None
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(
-                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                 "--format=csv,noheader,nounits", "-lms", "50"],
-                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
+            import pynvml
+            pynvml.nvmlInit()
+            idx = self.index
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            if vis and vis.split(",")[idx].strip().isdigit():
+                idx = int(vis.split(",")[idx])
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.nv = pynvml
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
-        except Exception:
-            self.proc = None
+        except Exception as e:          # no NVML: reported as unavailable, never faked
+            self.err = repr(e)
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.lines.append(line.strip())
+    def _run(self):
+        nv, h = self.nv, self.h
+        while not self.stop:
+            if self.active:
+                try:
+                    mhz = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+                    rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                    self.samples.append((mhz, rs))
+                except Exception as e:
+                    self.err = repr(e)
+                time.sleep(0.0005)
+            else:
+                time.sleep(0.0002)
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except Exception:
-                self.proc.kill()
+        self.stop = True
 
     def summary(self):
-        sm, mx, reasons = [], None, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
-            f = [x.strip() for x in ln.split(",")]
-            if len(f) < 9:
-                continue
-            try:
-                if float(f[8]) < 50:          # keep samples taken under load only
-                    continue
-                sm.append(float(f[1]))
-                mx = float(f[2])
-            except ValueError:
-                continue
-            for nm, v in zip(names, f[4:8]):
-                if v.lower() == "active":
-                    reasons.add(nm)
-        if not sm:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sm)}
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"],
+                    "samples": 0, "error": self.err}
+        reasons = sorted({nm for _, rs in self.samples for nm, b in self.BITS.items() if rs & b})
+        return {"sm_mhz": statistics.median(m for m, _ in self.samples), "sm_max_mhz": self.max_mhz,
+                "sm_min_mhz": min(m for m, _ in self.samples), "reasons": reasons,
+                "samples": len(self.samples), "source": "NVML, polled during the timed region"}
 
 
 def cpu_baseline(spec, bound, eps, seconds):
@@ -302,6 +305,7 @@ def run_ours(args):
         dist.barrier()
     torch.cuda.synchronize()
     t_wall0 = time.perf_counter()
+    clk.active = True
     for i in range(args.steps):
         ev[i][0].record(stream)
         r = compress_once()
@@ -309,17 +313,12 @@ def run_ours(args):
         decompress_once(r)
         ev[i][2].record(stream)
     torch.cuda.synchronize()
+    clk.active = False
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     t_wall = time.perf_counter() - t_wall0
     launches = pk.launch_count() - launches0
-    t_hold = time.perf_counter()
-    while len(clk.lines) < 4 and time.perf_counter() - t_hold < 2.0:
-        for _ in range(10):
-            rr = compress_once()
-            decompress_once(rr)
-        torch.cuda.synchronize()
     clk.__exit__(None, None, None)
     tc = [ev[i][0].elapsed_time(ev[i][1]) for i in range(args.steps)]
     td = [ev[i][1].elapsed_time(ev[i][2]) for i in range(args.steps)]

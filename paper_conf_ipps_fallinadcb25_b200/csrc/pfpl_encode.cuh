@@ -22,8 +22,12 @@
 // arena, so a slow look-back only delays the IO warp.
 // Thread t of the compute warps owns elements 32t..32t+31, so its 32 bits of
 // each bit plane are one aligned word of the shuffled chunk.
-// Arena slice of a chunk: [pos, pos + ZPRE + n1) with Z1 at pos + ZPRE and
-// M4 | Z4 | Z3 | Z2 packed immediately before it (section order of R16).
+// Arena slice of a chunk at pos: Z1 at [pos, pos + n1); the prefix M4 | Z4 | Z3 | Z2
+// (section order of R16) ends at pos + a16(n1) + PRE3 + n2, with Z2 at a fixed
+// offset PRE3 past Z1 (so all warps can scatter it before n3/n4 are known) and
+// M4 | Z4 | Z3 packed immediately before Z2.  A slice is reserved for the worst
+// case (a16(n1) + ZPRE) but occupies only a16(n1) + a16(PRE3 + n2): on smooth
+// data the prefix is a few dozen bytes, so the arena holds many chunks.
 #pragma once
 #include <cuda.h>
 #include "pfpl_device.cuh"
@@ -32,14 +36,15 @@ namespace pfpl {
 
 constexpr int NIN = 2;               // input stages (TMA ring)
 constexpr int DATAB = 16384;         // bytes per chunk
-constexpr int ZPRE = 2352;           // >= 4 + 32 + 256 + 2048, multiple of 16
+constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
+constexpr int ZPRE = 2352;           // >= PRE3 + 2048 (Z2 at most), multiple of 16
 constexpr int NQ = 8;                // IO queue depth
 constexpr int ARENA = 18752;         // circular payload arena (bytes, multiple of 16)
 
 // hand-off from the compute warps to the IO warp, one per chunk
 struct QEntry {
     unsigned long long c;
-    uint32_t start, stored, raw, rend;
+    uint32_t start, plen, z1, stored, raw, rend;   // prefix at start (plen bytes), Z1 at z1
 };
 
 struct EncShared {
@@ -91,6 +96,33 @@ __device__ __forceinline__ void scatter_marked(uint8_t* z, uint32_t o, uint32_t 
     if (H & 0x80000000u) z[o + (rk >> 24)] = (uint8_t)(w >> 24);
 }
 
+// copy len bytes from shared memory to global memory, any alignment on either
+// side: 16-byte aligned stores for the body (coalesced even for
+// unaligned compressed data), byte stores for the head and the tail.  Reads up
+// to 20 bytes past src + len (inside the arena's padding).
+__device__ __forceinline__ void warp_copy_s2g(uint8_t* o, const uint8_t* src, uint32_t len, int lane) {
+    const uint32_t mis = (uint32_t)((uintptr_t)o & 15u);
+    uint32_t head = (16u - mis) & 15u;
+    if (head > len) head = len;
+    const uint32_t body = (len - head) >> 4;
+    const uint32_t tail0 = head + (body << 4);
+    if ((uint32_t)lane < head) o[lane] = src[lane];
+    if ((uint32_t)lane < len - tail0) o[tail0 + lane] = src[tail0 + lane];
+    for (uint32_t j = lane; j < body; j += 32) {
+        const uint8_t* sp = src + head + (j << 4);
+        const uint32_t a = smem_u32(sp) & 3u;
+        const uint32_t* sw = (const uint32_t*)(sp - a);
+        const uint32_t w0 = sw[0], w1 = sw[1], w2 = sw[2], w3 = sw[3], w4 = sw[4];
+        const uint32_t sh = a * 8u;
+        uint4 v;
+        v.x = __funnelshift_r(w0, w1, sh);
+        v.y = __funnelshift_r(w1, w2, sh);
+        v.z = __funnelshift_r(w2, w3, sh);
+        v.w = __funnelshift_r(w3, w4, sh);
+        *(uint4*)(o + head + (j << 4)) = v;
+    }
+}
+
 // ---------------------------------------------------------------------------
 // bit shuffle + level-1 zero-byte elimination for one chunk.
 // KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
@@ -105,9 +137,11 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
 // Arena slice for a chunk with n1 Z1 bytes: every compute warp derives the same
 // position from S.head (advanced by warp 0 only after the Z1 scatter) and waits
 // only if the IO warp lags by more than the arena's capacity.
-__device__ __forceinline__ uint32_t slice_bytes(uint32_t n1) { return (ZPRE + n1 + 15u) & ~15u; }
+__device__ __forceinline__ uint32_t a16(uint32_t x) { return (x + 15u) & ~15u; }
+// bytes a slice occupies once n2 is known
+__device__ __forceinline__ uint32_t slice_bytes(uint32_t n1, uint32_t n2) { return a16(n1) + a16(PRE3 + n2); }
 __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
-    const uint32_t R = slice_bytes(n1);
+    const uint32_t R = a16(n1) + ZPRE;                      // worst case
     const uint32_t head0 = S.head;
     uint32_t head = head0;
     const uint32_t p0 = head % ARENA;
@@ -265,14 +299,6 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const QEntry e = S.q[slot];
             if (e.c >= C) break;
             const uint64_t c = e.c;
-            // lag behind the compute warps by up to one entry (bounded, so a slice
-            // that fills the arena cannot deadlock): by then the predecessors of
-            // chunk c have almost always published their aggregates
-            {
-                const uint32_t nb = smem_u32(&S.mq_full[(k + 1) % NQ]);
-                const uint32_t np = ((k + 1) / NQ) & 1u;
-                for (int tries = 0; tries < 16 && !mbar_test(nb, np); ++tries) __nanosleep(256);
-            }
             const uint32_t stored = e.stored, start = e.start;
             const bool israw = e.raw != 0;
             // ---- decoupled look-back ----
@@ -283,10 +309,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     const int64_t idx = look - lane;
                     uint64_t val = 0, flag = LB_P;
                     if (idx >= 0) {
-                        // the predecessor may still be in flight: back off so the
-                        // polling does not steal issue slots from the compute warps
+                        // the predecessor may still be in flight: back off a little so
+                        // the polling does not steal issue slots from the compute warps
+                        // (capped well below one chunk's encode time, ~2 us per CTA)
                         const uint64_t t0 = globaltimer();
-                        for (uint32_t ns = 256;; ns = ns < 8192 ? 2 * ns : ns) {
+                        for (uint32_t ns = 64;; ns = ns < 512 ? 2 * ns : ns) {
                             const uint64_t d = ld_relaxed(&p.status[idx]);
                             flag = ((uint32_t)(d >> 48) == p.epoch) ? ((d >> 46) & 3u) : 0u;
                             if (flag) { val = d & LB_VAL; break; }
@@ -312,7 +339,6 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 if (c == 0 && p.write_header) write_header(p.out, p, qc);
             }
             if (dst + stored <= p.cap) {
-                const uint8_t* src = arena + start;
                 if (israw) {
                     // raw chunk (R17): stage the original bytes in this chunk's
                     // arena slice (always large enough: slice >= payload >= raw bytes)
@@ -322,29 +348,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     for (uint32_t i = (stored / 16) * 4 + lane; i < stored / 4; i += 32)
                         ((uint32_t*)stg)[i] = ((const uint32_t*)g)[i];
                     __syncwarp();
-                }
-                // 16-byte aligned stores for the body (coalesced even for
-                // unaligned compressed data), bytes for the head and tail
-                uint8_t* o = p.out + dst;
-                const uint32_t mis = (uint32_t)((uintptr_t)o & 15u);
-                uint32_t head = (16u - mis) & 15u;
-                if (head > stored) head = stored;
-                const uint32_t body = (stored - head) >> 4;
-                const uint32_t tail0 = head + (body << 4);
-                if ((uint32_t)lane < head) o[lane] = src[lane];
-                if ((uint32_t)lane < stored - tail0) o[tail0 + lane] = src[tail0 + lane];
-                for (uint32_t j = lane; j < body; j += 32) {
-                    const uint8_t* sp = src + head + (j << 4);
-                    const uint32_t a = smem_u32(sp) & 3u;
-                    const uint32_t* sw = (const uint32_t*)(sp - a);
-                    const uint32_t w0 = sw[0], w1 = sw[1], w2 = sw[2], w3 = sw[3], w4 = sw[4];
-                    const uint32_t sh = a * 8u;
-                    uint4 v;
-                    v.x = __funnelshift_r(w0, w1, sh);
-                    v.y = __funnelshift_r(w1, w2, sh);
-                    v.z = __funnelshift_r(w2, w3, sh);
-                    v.w = __funnelshift_r(w3, w4, sh);
-                    *(uint4*)(o + head + (j << 4)) = v;
+                    warp_copy_s2g(p.out + dst, arena + start, stored, lane);
+                } else {
+                    // payload = prefix (M4 | Z4 | Z3 | Z2) then Z1 (R16)
+                    warp_copy_s2g(p.out + dst, arena + start, e.plen, lane);
+                    warp_copy_s2g(p.out + dst + e.plen, arena + e.z1, stored - e.plen, lane);
                 }
             }
             __syncwarp();
@@ -470,10 +478,10 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             n1 = tot_l + tot_h;
             head = slice_start(S, n1, lane);
         }
-        uint8_t* const z1 = arena + head % ARENA + ZPRE;
+        uint8_t* const z1 = arena + head % ARENA;
         PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
         named_sync(1, NTC);    // Z1 and M1 complete
-        if (tid == 0) S.head = head + slice_bytes(n1);
+        uint8_t* const z2 = z1 + a16(n1) + PRE3;
 
         // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 + Z2), P:131 ----
         const int slot = it % NQ;
@@ -511,8 +519,8 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 if (w < warp) base += v;
                 n2 += v;
             }
+            if (tid == 0) S.head = head + slice_bytes(n1, n2);
             if (cnt2) {
-                uint8_t* z2 = z1 - n2;
                 uint32_t o = base + inc - cnt2;
 #pragma unroll
                 for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
@@ -535,7 +543,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const bool dif = m3 != pm3;
             const uint32_t M4 = __ballot_sync(PFPL_FULL, dif);
             const uint32_t n4 = __popc(M4);
-            uint8_t* z3 = z1 - n2 - n3;
+            uint8_t* z3 = z2 - n3;
             scatter_word(z3, scatter_word(z3, inc3 - cnt3, v.x, h0), v.y, h1);
             uint8_t* z4 = z3 - n4;
             if (dif) z4[__popc(M4 & ((1u << lane) - 1u))] = (uint8_t)m3;
@@ -554,7 +562,9 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 e.stored = stored;
                 e.raw = israw ? 1u : 0u;
                 e.start = israw ? head % ARENA : (uint32_t)(z4 - 4 - arena);
-                e.rend = head + slice_bytes(n1);
+                e.plen = 4 + n4 + n3 + n2;
+                e.z1 = head % ARENA;
+                e.rend = head + slice_bytes(n1, n2);
                 mbar_arrive(smem_u32(&S.mq_full[slot]));
             }
         }
