@@ -360,7 +360,7 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     const int grid = decode_grid(dtype, mode, ms, nchunks);
     CK(launch_decode(dtype, mode, ms, p, grid, s));
     g_launches += 1;
-    sc->ticket_val += nchunks + (uint64_t)grid * (uint64_t)decode_tickets_per_cta();
+    sc->ticket_val += (uint64_t)grid * (uint64_t)decode_tickets_per_cta();   // decoder: no tickets
     return PFPL_OK;
 }
 

@@ -172,15 +172,20 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
 
     if (warp == NWC) {
         // =========================== IO warp ===========================
-        unsigned long long tnext = 0;
+        // static round-robin assignment (chunk c = blockIdx.x + k * gridDim.x): the
+        // offsets are known up front (size_scan_kernel), so no ticket atomics sit on
+        // the IO warp's critical path, and the next chunk's table entries are loaded
+        // one iteration ahead
         uint32_t head = 0;
-        if (lane == 0) tnext = atomicAdd(p.ticket, 1ull) - p.ticket_base;
-        for (uint32_t k = 0;; ++k) {
+        const uint64_t G = gridDim.x;
+        uint64_t c = blockIdx.x;
+        uint32_t size_n = 0;
+        uint64_t excl_n = 0;
+        if (c < C) { size_n = p.table[c]; excl_n = p.offs[c]; }
+        for (uint32_t k = 0;; ++k, c += G) {
             const int slot = k % NQD;
-            const unsigned long long c = __shfl_sync(PFPL_FULL, tnext, 0);
-            if (lane == 0) tnext = atomicAdd(p.ticket, 1ull) - p.ticket_base;
             if (c >= C) {
-                mbar_wait_wd(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
+                mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
                 if (lane == 0) {
                     S.q[slot].c = c;
                     mbar_arrive(smem_u32(&S.full[slot]));
@@ -188,8 +193,9 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 break;
             }
             // d1: chunk offset from the size-table prefix sum (size_scan_kernel)
-            const uint32_t size = p.table[c];
-            const uint64_t excl = p.offs[c];
+            const uint32_t size = size_n;
+            const uint64_t excl = excl_n;
+            if (c + G < C) { size_n = p.table[c + G]; excl_n = p.offs[c + G]; }
             const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
             const uint32_t rawb = m * S_;
             uint32_t bad = 0;
@@ -216,7 +222,9 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             }
             const uint32_t pos = head % RING;
             head += R;
-            mbar_wait_wd(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
+            // the IO warp runs up to NQD chunks ahead: waiting here is the common
+            // case, so sleep between polls instead of spinning on the issue port
+            mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
             // bulk copy of the aligned superset, never past the last 16-byte
             // boundary of the stream; the remainder by the lanes
             const uint8_t* a0 = g - delta;
@@ -431,18 +439,33 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
 
         // ---- dequantize into swizzled rows ----
         if (m == CW) {
+            auto emit = [&](auto dqf) {
 #pragma unroll
-            for (int i = 0; i < 2 * S_; ++i) {
-                T x[16 / S_];
+                for (int i = 0; i < 2 * S_; ++i) {
+                    T x[16 / S_];
 #pragma unroll
-                for (int k = 0; k < 16 / S_; ++k)
-                    x[k] = fastdq ? (T)q.abs_dq_fast((uint32_t)(carry + dq[i * (16 / S_) + k]), c23)
-                                  : dequantize<T, MODE>(q, (W)(carry + dq[i * (16 / S_) + k]), raw);
-                uint4 v;
-                memcpy(&v, x, 16);
-                const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
-                *(uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4)) = v;
+                    for (int k = 0; k < 16 / S_; ++k) x[k] = dqf((W)(carry + dq[i * (16 / S_) + k]));
+                    uint4 v;
+                    memcpy(&v, x, 16);
+                    const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                    *(uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4)) = v;
+                }
+            };
+            bool done = false;
+            if constexpr (sizeof(T) == 4 && MODE == MODE_ABS) {
+                if (fastdq) {
+                    // all words of this thread are bins (the common case): no raw-word select
+                    W wor = 0;
+#pragma unroll
+                    for (int i = 0; i < 32; ++i) wor |= (W)(carry + dq[i]);
+                    if (wor < 0x00800000u)
+                        emit([&](W w) { return (T)q.abs_dq_bins((uint32_t)w, c23); });
+                    else
+                        emit([&](W w) { return (T)q.abs_dq_fast((uint32_t)w, c23); });
+                    done = true;
+                }
             }
+            if (!done) emit([&](W w) { return dequantize<T, MODE>(q, w, raw); });
             fence_proxy_async();
             named_sync(1, NTC);    // staging complete
             if (tid == 0) {

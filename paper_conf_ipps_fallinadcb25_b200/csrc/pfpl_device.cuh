@@ -172,6 +172,19 @@ template <> struct QF<float> {
         asm("mad.lo.u32 %0, %1, 1, 0x4B000000;" : "=r"(rawb) : "r"(f2u(v)));
         return ok ? z : rawb;
     }
+    // fast-path biased word: same as abs_qb(v) whenever the value is quantizable;
+    // `ok` accumulates both checks of abs_qb (two chained FSETP.AND, no select and
+    // no raw word); if it ends false the caller redoes the words with abs_qb.
+    __device__ __forceinline__ uint32_t abs_qf(float v, bool& ok) const {
+        float s = v * b;
+        float t = s + 12582912.0f;
+        float rb = t - 12582912.0f;
+        float vr = rb * c;
+        float diff = fabsf(v - vr);
+        ok = ok && (fabsf(rb) < 4194304.0f) && (diff <= a);
+        const float w2 = __fmaf_rn(rb, 2.0f, 0.5f);
+        return f2u(fabsf(w2) + 8388607.5f);
+    }
     __device__ __forceinline__ float abs_dq(uint32_t w) const {
         return w < 0x00800000u ? __int2float_rn(unzz(w)) * c : u2f(w);
     }
@@ -182,6 +195,12 @@ template <> struct QF<float> {
         const float f = u2f((w + 0x96000001u) >> 1);
         const float mag = __fmaf_rn(f, c, -c23);
         return u2f(selp_u32(f2u(mag) ^ (w * 0x80000000u), w, w < 0x00800000u));
+    }
+    // abs_dq_fast for a word known to be a bin (w < 2^23)
+    __device__ __forceinline__ float abs_dq_bins(uint32_t w, float c23) const {
+        const float f = u2f((w + 0x96000001u) >> 1);
+        const float mag = __fmaf_rn(f, c, -c23);
+        return u2f(f2u(mag) ^ (w * 0x80000000u));
     }
     // REL: a = c_lo, b = w, c = inv_w.  log-space bin (R5), conservative
     // 1-ulp-shrunk check (R7), sign+bin in the negative-NaN payload (R10),
@@ -288,8 +307,6 @@ __device__ __forceinline__ typename Tr<T>::W quantize_b(const QF<T>& q, T v, boo
     }
     return quantize<T, MODE>(q, v, raw);
 }
-template <typename T, int MODE> struct QBias { static constexpr uint64_t v = 0; };
-template <> struct QBias<float, MODE_ABS> { static constexpr uint64_t v = 0x4B000000u; };
 
 template <typename T, int MODE>
 __device__ __forceinline__ T dequantize(const QF<T>& q, typename Tr<T>::W w, bool raw);
@@ -534,6 +551,18 @@ __device__ __forceinline__ void mbar_wait_wd(uint32_t a, uint32_t parity, uint32
     const uint64_t t0 = globaltimer();
     for (;;) {
         if (mbar_try_hint(a, parity, hint_ns)) return;
+        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(site, parity);
+    }
+}
+// poll with a sleep between tries: for waits that are the common case and whose
+// latency does not matter (a producer running ahead of its consumers)
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t a, uint32_t parity, uint32_t site,
+                                                uint32_t ns = 256) {
+    if (mbar_try(a, parity)) return;
+    const uint64_t t0 = globaltimer();
+    for (;;) {
+        __nanosleep(ns);
+        if (mbar_try(a, parity)) return;
         if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(site, parity);
     }
 }

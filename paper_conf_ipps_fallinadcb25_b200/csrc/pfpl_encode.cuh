@@ -304,24 +304,29 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             // ---- decoupled look-back ----
             uint64_t excl = 0;
             if (c > 0) {
+                // windows of 32 predecessors, lane l reads chunk look-l; the window is
+                // re-read (after a short sleep, so polling costs the compute warps
+                // almost no issue slots) until every chunk up to the first inclusive
+                // prefix has published
                 int64_t look = (int64_t)c - 1;
+                const uint64_t t0 = globaltimer();
                 for (;;) {
                     const int64_t idx = look - lane;
-                    uint64_t val = 0, flag = LB_P;
+                    uint64_t val = 0;
+                    uint32_t flag = (uint32_t)LB_P;               // before chunk 0: prefix 0
                     if (idx >= 0) {
-                        // the predecessor may still be in flight: back off a little so
-                        // the polling does not steal issue slots from the compute warps
-                        // (capped well below one chunk's encode time, ~2 us per CTA)
-                        const uint64_t t0 = globaltimer();
-                        for (uint32_t ns = 64;; ns = ns < 512 ? 2 * ns : ns) {
-                            const uint64_t d = ld_relaxed(&p.status[idx]);
-                            flag = ((uint32_t)(d >> 48) == p.epoch) ? ((d >> 46) & 3u) : 0u;
-                            if (flag) { val = d & LB_VAL; break; }
-                            if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x12, (uint32_t)idx);
-                            __nanosleep(ns);
-                        }
+                        const uint64_t d = ld_relaxed(&p.status[idx]);
+                        flag = ((uint32_t)(d >> 48) == p.epoch) ? (uint32_t)((d >> 46) & 3u) : 0u;
+                        val = d & LB_VAL;
                     }
                     const uint32_t pm = __ballot_sync(PFPL_FULL, flag == LB_P);
+                    const uint32_t nr = __ballot_sync(PFPL_FULL, flag == 0u);
+                    const uint32_t need = pm ? ((pm & (0u - pm)) << 1) - 1u : PFPL_FULL;
+                    if (nr & need) {
+                        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x12, (uint32_t)look);
+                        __nanosleep(400);
+                        continue;
+                    }
                     if (pm) {
                         const int first = __ffs(pm) - 1;
                         excl += warp_sum64(lane <= first ? val : 0ull);
@@ -392,7 +397,39 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         {
             // biased words (quantize_b): q + bias; the bias cancels in q[i] - q[i-1]
             W qprev = (W)qbias;
-            if (m == CW) {
+            bool done = false;
+            if constexpr (sizeof(T) == 4 && (MODE == MODE_ABS || MODE == MODE_NOA)) {
+                if (m == CW && !raw) {
+                    // fast path: no per-element select or raw word; the
+                    // checks of all 32 values accumulate into one predicate
+                    uint32_t zp = (uint32_t)qbias, orw = 0u;
+                    // 8 independent predicate chains (a single chain would serialise
+                    // 64 dependent FSETPs per thread)
+                    bool ok[8] = {true, true, true, true, true, true, true, true};
+                    if (tid > 0) {
+                        const int r = tid - 1;
+                        zp = q.abs_qf(*(const float*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 12), ok[7]);
+                    }
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const uint4 v = *(const uint4*)(buf + tid * 128 + (((i & 7) ^ (tid & 7)) << 4));
+                        bool* o = ok + 4 * (i & 1);
+                        const uint32_t z0 = q.abs_qf(u2f(v.x), o[0]), z1 = q.abs_qf(u2f(v.y), o[1]);
+                        const uint32_t z2 = q.abs_qf(u2f(v.z), o[2]), z3 = q.abs_qf(u2f(v.w), o[3]);
+                        const uint32_t r0 = rcode<MSR>(z0 - zp), r1 = rcode<MSR>(z1 - z0);
+                        const uint32_t r2 = rcode<MSR>(z2 - z1), r3 = rcode<MSR>(z3 - z2);
+                        zp = z3;
+                        orw |= r0 | r1;
+                        orw |= r2 | r3;
+                        lo[4 * i] = r0; lo[4 * i + 1] = r1; lo[4 * i + 2] = r2; lo[4 * i + 3] = r3;
+                    }
+                    done = __all_sync(PFPL_FULL, ok[0] && ok[1] && ok[2] && ok[3] && ok[4] && ok[5] &&
+                                                     ok[6] && ok[7]);
+                    orv = (W)orw;
+                }
+            }
+            if (done) {
+            } else if (m == CW) {
                 if (tid > 0) {
                     T pv;
                     if (sizeof(T) == 4) {
