@@ -323,8 +323,10 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     const uint32_t nr = __ballot_sync(PFPL_FULL, flag == 0u);
                     const uint32_t need = pm ? ((pm & (0u - pm)) << 1) - 1u : PFPL_FULL;
                     if (nr & need) {
+                        // a predecessor is still being encoded (typically ~1 chunk time):
+                        // the IO warp's latency is hidden by the arena, so poll rarely
                         if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x12, (uint32_t)look);
-                        __nanosleep(400);
+                        __nanosleep(1500);
                         continue;
                     }
                     if (pm) {
