@@ -41,9 +41,11 @@ def lib():
     """Load libpfpl.so (built in-tree by __graft_entry__.build())."""
     global _lib
     if _lib is None:
-        if not os.path.exists(_build.LIB):
-            raise PFPLError(-6, f"{_build.LIB} is missing; run __graft_entry__.build()")
-        L = ctypes.CDLL(_build.LIB)
+        # PFPL_LIB names an in-tree tuning variant (tools/variants.sh); default libpfpl.so
+        path = os.path.join(os.path.dirname(_build.LIB), os.environ.get("PFPL_LIB", "libpfpl.so"))
+        if not os.path.exists(path):
+            raise PFPLError(-6, f"{path} is missing; run __graft_entry__.build()")
+        L = ctypes.CDLL(path)
         vp, u64, i32, dbl = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_int, ctypes.c_double
         pu64 = ctypes.POINTER(ctypes.c_uint64)
         sig = {

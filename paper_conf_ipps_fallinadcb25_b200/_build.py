@@ -45,10 +45,15 @@ def needs_build() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS)
 
 
-def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count() or 8) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count() or 8,
+          out: str | None = None, extra: list | None = None) -> str:
+    """Compile libpfpl.so (or, for tuning experiments, a variant library `out`
+    built with `extra` nvcc flags, e.g. -DPFPL_ENC_NIN=1)."""
+    lib = out or LIB
+    extra = list(extra or [])
+    if not force and not extra and out is None and not needs_build():
         return LIB
-    bdir = os.path.join(ROOT, "build")
+    bdir = os.path.join(ROOT, "build" if not extra else "build_" + os.path.basename(lib).replace(".so", ""))
     os.makedirs(bdir, exist_ok=True)
     jobs_ = []
     for src in SRCS:
@@ -62,7 +67,7 @@ def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count()
     while pending or running:
         while pending and len(running) < max(1, jobs):
             src, obj, defs = pending.pop(0)
-            cmd = [nvcc(), *NVCC_FLAGS, *defs, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
+            cmd = [nvcc(), *NVCC_FLAGS, *extra, *defs, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
             log = open(obj + ".log", "w")
             running.append((subprocess.Popen(cmd, stdout=log, stderr=subprocess.STDOUT), cmd, obj))
         p, cmd, obj = running.pop(0)
@@ -72,13 +77,17 @@ def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count()
             raise RuntimeError("nvcc failed: " + " ".join(cmd) + "\n" + open(obj + ".log").read())
         if verbose:
             print(open(obj + ".log").read())
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     subprocess.run([nvcc(), "-shared", "-gencode", "arch=compute_100a,code=sm_100a", *objs,
                     "-o", tmp], check=True)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    build(force=True, verbose=True)
-    print(LIB)
+    import sys
+    if len(sys.argv) > 2:      # _build.py OUT.so -DFLAG ...   (tuning variants)
+        print(build(force=True, out=os.path.join(PKG, sys.argv[1]), extra=sys.argv[2:]))
+    else:
+        build(force=True, verbose=True)
+        print(LIB)

@@ -34,12 +34,24 @@
 
 namespace pfpl {
 
-constexpr int NIN = 2;               // input stages (TMA ring)
+#ifndef PFPL_ENC_NIN
+#define PFPL_ENC_NIN 1
+#endif
+#ifndef PFPL_ENC_MINB
+#define PFPL_ENC_MINB 5
+#endif
+#ifndef PFPL_ENC_ARENA
+#define PFPL_ENC_ARENA 18752
+#endif
+constexpr int NIN = PFPL_ENC_NIN;    // input stages (TMA ring)
 constexpr int DATAB = 16384;         // bytes per chunk
 constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 constexpr int ZPRE = 2352;           // >= PRE3 + 2048 (Z2 at most), multiple of 16
-constexpr int NQ = 8;                // IO queue depth
-constexpr int ARENA = 18752;         // circular payload arena (bytes, multiple of 16)
+#ifndef PFPL_ENC_NQ
+#define PFPL_ENC_NQ 8
+#endif
+constexpr int NQ = PFPL_ENC_NQ;      // IO queue depth
+constexpr int ARENA = PFPL_ENC_ARENA; // circular payload arena (bytes, multiple of 16)
 
 // hand-off from the compute warps to the IO warp, one per chunk
 struct QEntry {
@@ -50,7 +62,7 @@ struct QEntry {
 struct EncShared {
     uint8_t m1[2048];
     uint8_t m2[256];
-    uint8_t wcnt[4][64];
+    uint8_t wcnt[128];               // per-warp per-plane Z1 counts, [warp * B + bit]
     uint32_t scan2[4];               // level-2 warp totals
     uint32_t head, tail;
     unsigned long long in_c[NIN];
@@ -60,7 +72,7 @@ struct EncShared {
 constexpr int ARENA_OFF = NIN * DATAB;
 constexpr int SHARED_OFF = ARENA_OFF + ARENA + 64;
 constexpr int ENC_SMEM = SHARED_OFF + (int)sizeof(EncShared);
-static_assert(ENC_SMEM <= 57344, "4 CTAs per SM need <= 56 KiB of shared memory each");
+static_assert(ENC_SMEM <= 233472 / PFPL_ENC_MINB - 1024, "PFPL_ENC_MINB CTAs per SM must fit in shared memory");
 static_assert(ZPRE + DATAB <= ARENA, "the arena must hold a worst-case chunk");
 
 __device__ __forceinline__ void put_u64(uint8_t* p, uint64_t v) {
@@ -188,13 +200,13 @@ __device__ __forceinline__ void rze1_count(uint32_t (&lo)[32], uint32_t (&hi)[32
             inc = warp_incl_scan(v, lane);
         }
         ex[g] = inc - v;
-        if (lane == 31) *(uint32_t*)&S.wcnt[warp][b0] = inc;
+        if (lane == 31) *(uint32_t*)&S.wcnt[warp * B + b0] = inc;
     }
     if (lane == 31) {
 #pragma unroll
-        for (int b0 = KL; b0 < 32; b0 += 4) *(uint32_t*)&S.wcnt[warp][b0] = 0u;
+        for (int b0 = KL; b0 < 32; b0 += 4) *(uint32_t*)&S.wcnt[warp * B + b0] = 0u;
 #pragma unroll
-        for (int b0 = 32 + KH; b0 < B; b0 += 4) *(uint32_t*)&S.wcnt[warp][b0] = 0u;
+        for (int b0 = 32 + KH; b0 < B; b0 += 4) *(uint32_t*)&S.wcnt[warp * B + b0] = 0u;
     }
 }
 
@@ -242,7 +254,7 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
     } while (0)
 
 template <typename T, int MODE, bool MSR>
-__global__ void __launch_bounds__(Tr<T>::NT + 32, 4)
+__global__ void __launch_bounds__(Tr<T>::NT + 32, PFPL_ENC_MINB)
 encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
     constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;
@@ -276,7 +288,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         if (smem_u32(smem) & 1023u) __trap();       // TMA SWIZZLE_128B needs 1024-byte alignment
         for (int s = 0; s < NIN; ++s) mbar_init(smem_u32(&S.full[s]), 1);
         for (int k = 0; k < NQ; ++k) {
-            mbar_init(smem_u32(&S.mq_full[k]), 1);
+            mbar_init(smem_u32(&S.mq_full[k]), NWC);     // every compute warp arrives
             mbar_init(smem_u32(&S.mq_empty[k]), 1);
         }
         S.head = 0;
@@ -497,8 +509,8 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             uint32_t myl = 0, myh = 0, tl = 0, th = 0;
 #pragma unroll
             for (int w = 0; w < NWC; ++w) {
-                const uint32_t a = S.wcnt[w][lane];
-                const uint32_t b = B == 64 ? S.wcnt[w][32 + lane] : 0u;
+                const uint32_t a = S.wcnt[w * B + lane];
+                const uint32_t b = B == 64 ? S.wcnt[w * B + 32 + lane] : 0u;
                 if (w < warp) { myl += a; myh += b; }
                 tl += a;
                 th += b;
@@ -567,7 +579,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
 
             // ---- levels 3 and 4 on the 256-byte M2, size, raw decision,
             // aggregate, hand-off: one duty warp, rotating so no warp is always late ----
-            if (warp != (int)(it % NWC)) continue;
+            if (warp != (int)(it % NWC)) {
+                // this warp's Z2 bytes are written: release them to the IO warp (the
+                // entry's phase completes only with the duty warp's arrival)
+                __syncwarp();
+                if (lane == 0) mbar_arrive(smem_u32(&S.mq_full[slot]));
+                continue;
+            }
             const uint2 v = ((const uint2*)S.m2)[lane];
             uint32_t pm2 = __shfl_up_sync(PFPL_FULL, v.y, 1);
             if (lane == 0) pm2 = 0;
@@ -608,11 +626,14 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             }
         }
     }
-    // end of work: tell the IO warp (queue position `it` gets a terminal entry)
-    if (tid == 0) {
+    // end of work: tell the IO warp (queue position `it` gets a terminal entry;
+    // all compute warps leave at the same `it` and each arrives once)
+    if (lane == 0) {
         const int slot = it % NQ;
-        mbar_wait_wd(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u, 0x16);
-        S.q[slot].c = ~0ull;
+        if (tid == 0) {
+            mbar_wait_wd(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u, 0x16);
+            S.q[slot].c = ~0ull;
+        }
         mbar_arrive(smem_u32(&S.mq_full[slot]));
     }
 }
