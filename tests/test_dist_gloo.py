@@ -70,6 +70,7 @@ def _worker(rank, world, port, bound, q):
             offs_ok = all(stream[p[3]:p[3] + len(p[1])] == p[1] and stream[p[4]:p[4] + len(p[2])] == p[2]
                           for p in parts)
             q.put((ok, offs_ok, parts[0][5] == len(full)))
+        dist.barrier()          # neither rank tears down the pair while the other still uses it
     finally:
         dist.destroy_process_group()
 
