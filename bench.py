@@ -191,6 +191,18 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def _traffic(config, bound):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of the encoder /
+    decoder, from the committed ncu --set full summary (profiles/traffic.json)"""
+    f = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "traffic.json")
+    try:
+        t = json.load(open(f))
+    except (OSError, ValueError):
+        return {}
+    e = t.get(f"{config}/{bound}", {})
+    return dict(e, source=t.get("source")) if e else {}
+
+
 def _config(spec, args, sample_rows=None):
     c = {"workload": f"{spec.name}, {args.bound.upper()} {args.eps:g}", "shape": list(spec.shape),
          "bound": args.bound, "eps": args.eps, "n": spec.n, "bytes": spec.nbytes,
@@ -339,13 +351,17 @@ def run_ours(args):
     enc_ms = statistics.median(tc)
     my_comp = comp_bytes if world == 1 else (4 * nch + r.payload.numel())
     algo = nbytes + my_comp                  # input read + stream written, per launch (this rank)
+    traffic = _traffic(args.config, args.bound)
     roof = {"bound": "hbm", "achieved": algo / (enc_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
-            "frac": algo / (enc_ms * 1e-3) / 1e9 / peak, "traffic": None,
+            "frac": algo / (enc_ms * 1e-3) / 1e9 / peak,
+            "traffic": traffic.get("encode") if world == 1 else None,
+            "traffic_source": traffic.get("source"), "algorithmic_bytes": algo,
             "kernel": "encode_kernel (compress step)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)" if peaks else "fallback 6.65 TB/s (B200_PROFILING.md)"}
     dec_ms = statistics.median(td)
     roof_dec = {"kernel": "decode_kernel", "achieved": algo / (dec_ms * 1e-3) / 1e9,
-                "frac": algo / (dec_ms * 1e-3) / 1e9 / peak}
+                "frac": algo / (dec_ms * 1e-3) / 1e9 / peak,
+                "traffic": traffic.get("decode") if world == 1 else None}
 
     # ---- end to end through the public API with host buffers (pinned) ----
     xh = x.cpu().pin_memory()

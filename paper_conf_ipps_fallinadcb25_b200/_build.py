@@ -63,6 +63,15 @@ def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count()
                       [f"-DPFPL_KIND={k}", f"-DPFPL_DT={d}", f"-DPFPL_MODE={m}"]))
     jobs_.sort(key=lambda j: 0 if j[2] else 1)      # long instantiation TUs first
     objs = [j[1] for j in jobs_]
+    # tuning variants: PFPL_VARIANT_ONLY="enc_0_0,dec_0_0" recompiles only those
+    # instantiations (plus the host files); the rest are linked from build/
+    only = os.environ.get("PFPL_VARIANT_ONLY")
+    if extra and only:
+        keep = set(only.split(","))
+        base = os.path.join(ROOT, "build")
+        objs = [o if (not j[2] or os.path.basename(o)[:-2] in keep) else os.path.join(base, os.path.basename(o))
+                for j, o in zip(jobs_, objs)]
+        jobs_ = [j for j in jobs_ if not j[2] or os.path.basename(j[1])[:-2] in keep]
     running, pending = [], list(jobs_)
     while pending or running:
         while pending and len(running) < max(1, jobs):

@@ -465,6 +465,26 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                     done = true;
                 }
             }
+            if constexpr (MODE == MODE_REL || sizeof(T) == 8) {
+                // long dequantizers (REL's pow2p, f64): stage the words, then dequantize
+                // them in place in a rolled loop (unrolled over 32 values the code
+                // overflows the instruction cache; see the encoder's TWO_PASS)
+                emit([&](W w) { T y; memcpy(&y, &w, sizeof(T)); return y; });
+#pragma unroll 1
+                for (int i = 0; i < 2 * S_; ++i) {
+                    const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                    uint4* const a = (uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4));
+                    uint4 v = *a;
+                    W w[16 / S_];
+                    T y[16 / S_];
+                    memcpy(w, &v, 16);
+#pragma unroll
+                    for (int k = 0; k < 16 / S_; ++k) y[k] = dequantize<T, MODE>(q, w[k], raw);
+                    memcpy(&v, y, 16);
+                    *a = v;
+                }
+                done = true;
+            }
             if (!done) emit([&](W w) { return dequantize<T, MODE>(q, w, raw); });
             fence_proxy_async();
             named_sync(1, NTC);    // staging complete

@@ -26,7 +26,7 @@
 // (section order of R16) ends at pos + a16(n1) + PRE3 + n2, with Z2 at a fixed
 // offset PRE3 past Z1 (so all warps can scatter it before n3/n4 are known) and
 // M4 | Z4 | Z3 packed immediately before Z2.  A slice is reserved for the worst
-// case (a16(n1) + ZPRE) but occupies only a16(n1) + a16(PRE3 + n2): on smooth
+// case (a16(n1) + a16(PRE3 + zroom(n1))) but occupies only a16(n1) + a16(PRE3 + n2): on smooth
 // data the prefix is a few dozen bytes, so the arena holds many chunks.
 #pragma once
 #include <cuda.h>
@@ -41,14 +41,16 @@ namespace pfpl {
 #define PFPL_ENC_MINB 5
 #endif
 #ifndef PFPL_ENC_ARENA
-#define PFPL_ENC_ARENA 18752
+#define PFPL_ENC_ARENA 16704
 #endif
 constexpr int NIN = PFPL_ENC_NIN;    // input stages (TMA ring)
 constexpr int DATAB = 16384;         // bytes per chunk
 constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
-constexpr int ZPRE = 2352;           // >= PRE3 + 2048 (Z2 at most), multiple of 16
 #ifndef PFPL_ENC_NQ
 #define PFPL_ENC_NQ 8
+#endif
+#ifndef PFPL_LB_NS
+#define PFPL_LB_NS 1500
 #endif
 constexpr int NQ = PFPL_ENC_NQ;      // IO queue depth
 constexpr int ARENA = PFPL_ENC_ARENA; // circular payload arena (bytes, multiple of 16)
@@ -73,7 +75,7 @@ constexpr int ARENA_OFF = NIN * DATAB;
 constexpr int SHARED_OFF = ARENA_OFF + ARENA + 64;
 constexpr int ENC_SMEM = SHARED_OFF + (int)sizeof(EncShared);
 static_assert(ENC_SMEM <= 233472 / PFPL_ENC_MINB - 1024, "PFPL_ENC_MINB CTAs per SM must fit in shared memory");
-static_assert(ZPRE + DATAB <= ARENA, "the arena must hold a worst-case chunk");
+static_assert(DATAB + 16 + ((PRE3 + 15) & ~15) <= ARENA, "the arena must hold a worst-case slice");
 
 __device__ __forceinline__ void put_u64(uint8_t* p, uint64_t v) {
 #pragma unroll
@@ -150,10 +152,17 @@ __device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
 // position from S.head (advanced by warp 0 only after the Z1 scatter) and waits
 // only if the IO warp lags by more than the arena's capacity.
 __device__ __forceinline__ uint32_t a16(uint32_t x) { return (x + 15u) & ~15u; }
+// room reserved for Z2: at most 2048 bytes, and never more than a non-raw chunk
+// can use (4 + n4 + n3 + n2 + n1 < 16384); a chunk whose n2 exceeds it is raw
+// (P:158), so its Z2 is not written.  A slice therefore never exceeds
+// 16400 + a16(PRE3) bytes, and a raw chunk's slice holds its 16384 staged bytes.
+__device__ __forceinline__ uint32_t zroom(uint32_t n1) { return min(2048u, (uint32_t)DATAB + 16u - a16(n1)); }
 // bytes a slice occupies once n2 is known
-__device__ __forceinline__ uint32_t slice_bytes(uint32_t n1, uint32_t n2) { return a16(n1) + a16(PRE3 + n2); }
+__device__ __forceinline__ uint32_t slice_bytes(uint32_t n1, uint32_t n2) {
+    return a16(n1) + a16(PRE3 + min(n2, zroom(n1)));
+}
 __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
-    const uint32_t R = a16(n1) + ZPRE;                      // worst case
+    const uint32_t R = a16(n1) + a16(PRE3 + zroom(n1));     // worst case
     const uint32_t head0 = S.head;
     uint32_t head = head0;
     const uint32_t p0 = head % ARENA;
@@ -254,7 +263,7 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
     } while (0)
 
 template <typename T, int MODE, bool MSR>
-__global__ void __launch_bounds__(Tr<T>::NT + 32, PFPL_ENC_MINB)
+__global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_ENC_MINB : 5)
 encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
     constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;
@@ -299,7 +308,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     __syncthreads();
     if (tid == 0) {
         for (int s = 0; s < NIN; ++s) issue(s, atomicAdd(p.ticket, 1ull) - p.ticket_base);
-        next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+        next = atomicAdd(p.ticket, 1ull);
     }
 
     if (warp == NWC) {
@@ -338,7 +347,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         // a predecessor is still being encoded (typically ~1 chunk time):
                         // the IO warp's latency is hidden by the arena, so poll rarely
                         if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x12, (uint32_t)look);
-                        __nanosleep(1500);
+                        __nanosleep(PFPL_LB_NS);
                         continue;
                     }
                     if (pm) {
@@ -442,8 +451,64 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     orv = (W)orw;
                 }
             }
+            // long quantizers (REL's log2p/pow2p/divisions, f64): quantize the stage in
+            // place in a rolled loop, then delta-code the words.  Fully unrolling them
+            // over 32 values overflows the instruction cache (ncu: no_instruction stalls
+            // were 42% of REL samples).
+            constexpr bool TWO_PASS = MODE == MODE_REL || sizeof(T) == 8;
+            if constexpr (TWO_PASS) {
+                if (m == CW) {
+                    uint8_t* const wbuf = smem + s * DATAB;
+                    T pv = (T)0;
+                    if (tid > 0) {
+                        if (lane == 0) {
+                            // the previous row belongs to another warp, which may
+                            // already have overwritten it: read the input again (L2)
+                            pv = ((const T*)p.in)[c * (uint64_t)CW + 32 * tid - 1];
+                        } else if (sizeof(T) == 4) {
+                            const int r = tid - 1;
+                            pv = *(const T*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 12);
+                        } else {
+                            const int r = 2 * tid - 1;
+                            pv = *(const T*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 8);
+                        }
+                    }
+                    __syncwarp();
+#pragma unroll 1
+                    for (int i = 0; i < 2 * S_; ++i) {
+                        const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                        uint4* const a = (uint4*)(wbuf + r * 128 + (((i & 7) ^ (r & 7)) << 4));
+                        uint4 v = *a;
+                        T x[16 / S_];
+                        W w[16 / S_];
+                        memcpy(x, &v, 16);
+#pragma unroll
+                        for (int k = 0; k < 16 / S_; ++k) w[k] = quantize_b<T, MODE>(q, x[k], raw);
+                        memcpy(&v, w, 16);
+                        *a = v;
+                    }
+                    if (tid > 0) qprev = quantize_b<T, MODE>(q, pv, raw);
+                    fence_proxy_async();      // the stage is refilled by TMA after the next barrier
+#pragma unroll
+                    for (int i = 0; i < 2 * S_; ++i) {
+                        const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                        const uint4 v = *(const uint4*)(buf + r * 128 + (((i & 7) ^ (r & 7)) << 4));
+                        W x[16 / S_];
+                        memcpy(x, &v, 16);
+#pragma unroll
+                        for (int k = 0; k < 16 / S_; ++k) {
+                            const W r2 = rcode<MSR>((W)(x[k] - qprev));
+                            qprev = x[k];
+                            orv |= r2;
+                            lo[i * (16 / S_) + k] = (uint32_t)r2;
+                            hi[i * (16 / S_) + k] = sizeof(W) == 8 ? (uint32_t)((uint64_t)r2 >> 32) : 0u;
+                        }
+                    }
+                    done = true;
+                }
+            }
             if (done) {
-            } else if (m == CW) {
+            } else if (!TWO_PASS && m == CW) {
                 if (tid > 0) {
                     T pv;
                     if (sizeof(T) == 4) {
@@ -498,8 +563,10 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         named_sync(1, NTC);    // counts visible; every row of stage s consumed
         if (tid == 0) {
             // refill stage s with the prefetched ticket; prefetch the next one
-            const unsigned long long t = next;
-            next = atomicAdd(p.ticket, 1ull) - p.ticket_base;
+            // (the raw ticket is kept: subtracting the base here would wait for the
+            // atomic's round trip right before the next barrier)
+            const unsigned long long t = next - p.ticket_base;
+            next = atomicAdd(p.ticket, 1ull);
             issue(s, t);
         }
         // Z1 offsets of this warp's segments: planes in decreasing bit order,
@@ -571,7 +638,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 n2 += v;
             }
             if (tid == 0) S.head = head + slice_bytes(n1, n2);
-            if (cnt2) {
+            if (cnt2 && n2 <= zroom(n1)) {        // else the chunk is raw (see zroom)
                 uint32_t o = base + inc - cnt2;
 #pragma unroll
                 for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
