@@ -24,8 +24,17 @@
 
 namespace pfpl {
 
+#ifndef PFPL_DEC_IO_NS
+#define PFPL_DEC_IO_NS 256
+#endif
 constexpr int NQD = 8;                 // chunks in flight per CTA (payload queue depth)
-constexpr int RING = 32768;            // circular payload ring (bytes, multiple of 16)
+#ifndef PFPL_DEC_RING
+#define PFPL_DEC_RING 24576
+#endif
+#ifndef PFPL_DEC_MINB
+#define PFPL_DEC_MINB 5
+#endif
+constexpr int RING = PFPL_DEC_RING;    // circular payload ring (bytes, multiple of 16)
 
 struct DecEntry {
     unsigned long long c;
@@ -45,7 +54,7 @@ constexpr int DOUT = 0;                // swizzled output staging (1024-aligned)
 constexpr int DRING = 16384;
 constexpr int DSH_OFF = DRING + RING + 64;
 constexpr int DEC_SMEM = DSH_OFF + (int)sizeof(DecShared);
-static_assert(DEC_SMEM <= 57344, "4 CTAs per SM need <= 56 KiB of shared memory each");
+static_assert(DEC_SMEM <= 233472 / PFPL_DEC_MINB - 1024, "PFPL_DEC_MINB CTAs per SM must fit in shared memory");
 
 __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t mbar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -144,7 +153,7 @@ __device__ __forceinline__ void dec1_gather(uint32_t (&lo)[32], uint32_t (&hi)[3
 __device__ __forceinline__ void set_err(int* err) { atomicExch(err, -4); }
 
 template <typename T, int MODE, bool MSR>
-__global__ void __launch_bounds__(Tr<T>::NT + 32, 4)
+__global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_DEC_MINB : 4)
 decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
     constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;
@@ -224,7 +233,7 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             head += R;
             // the IO warp runs up to NQD chunks ahead: waiting here is the common
             // case, so sleep between polls instead of spinning on the issue port
-            mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
+            mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21, PFPL_DEC_IO_NS);
             // bulk copy of the aligned superset, never past the last 16-byte
             // boundary of the stream; the remainder by the lanes
             const uint8_t* a0 = g - delta;
