@@ -55,7 +55,7 @@ unsigned int* watchdog_ptr() {
     return g_wd_dev;
 }
 
-constexpr int kMinmaxBlocks = 592;
+constexpr int kMinmaxBlocks = 1184;   // 8 CTAs of 256 threads per SM
 
 int cuda_fail(cudaError_t e) {
     g_last_cuda = (int)e;

@@ -25,7 +25,7 @@
 namespace pfpl {
 
 #ifndef PFPL_DEC_IO_NS
-#define PFPL_DEC_IO_NS 256
+#define PFPL_DEC_IO_NS 1024       // the IO warp runs up to 8 chunks ahead: poll rarely
 #endif
 constexpr int NQD = 8;                 // chunks in flight per CTA (payload queue depth)
 #ifndef PFPL_DEC_RING

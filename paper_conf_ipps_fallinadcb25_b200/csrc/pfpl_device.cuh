@@ -116,6 +116,93 @@ PFPL_HD double pow2p_f64(double y) {
     return p * u2d((uint64_t)(ki + 1023) << 52);
 }
 
+// Device forms of log2p_f32 / pow2p_f32 with the same bits and no XU-pipe
+// conversions: for an integer-valued float or int |x| < 2^22, x + 1.5*2^23 has bits
+// 0x4B400000 + x, which replaces (float)e, rintf and (int)k exactly.
+// pow2p: for |y| >= 2^22 both forms of k are beyond +-127 (or NaN/inf), so both
+// return the same inf / 0.
+__device__ __forceinline__ float i2f_small(int e) { return u2f(0x4B400000u + (uint32_t)e) - 12582912.0f; }
+__device__ __forceinline__ float log2p_f32_d(float a) {
+    uint32_t u = f2u(a);
+    int e = (int)((u >> 23) & 0xFFu) - 127;
+    float m = u2f((u & 0x007FFFFFu) | 0x3F800000u);
+    if (m > u2f(0x3FB504F3u)) { m = m * 0.5f; e = e + 1; }
+    float t = (m - 1.0f) / (m + 1.0f);
+    float t2 = t * t;
+    float p = u2f(0x3ED30BB1u);
+    p = p * t2; p = p + u2f(0x3F13BB63u);
+    p = p * t2; p = p + u2f(0x3F76384Fu);
+    p = p * t2; p = p + u2f(0x4038AA3Bu);
+    float r = t * p;
+    return i2f_small(e) + r;
+}
+__device__ __forceinline__ float pow2p_f32_d(float y) {
+    const float tk = y + 12582912.0f;
+    float k = tk - 12582912.0f;
+    float f = y - k;
+    float p = u2f(0x377FE5FEu);
+    p = p * f; p = p + u2f(0x39218489u);
+    p = p * f; p = p + u2f(0x3AAEC3FFu);
+    p = p * f; p = p + u2f(0x3C1D955Bu);
+    p = p * f; p = p + u2f(0x3D635847u);
+    p = p * f; p = p + u2f(0x3E75FDF0u);
+    p = p * f; p = p + u2f(0x3F317218u);
+    p = p * f; p = p + 1.0f;
+    if (!(k <= 127.0f)) return u2f(0x7F800000u);
+    if (k < -126.0f) return 0.0f;
+    const int ki = (int)(f2u(tk) - 0x4B400000u);
+    return p * u2f((uint32_t)(ki + 127) << 23);
+}
+
+// f64 forms: x + 1.5*2^52 has bits 0x4338000000000000 + x for integer |x| < 2^51
+__device__ __forceinline__ double i2d_small(long long e) {
+    return u2d(0x4338000000000000ull + (uint64_t)e) - 6755399441055744.0;
+}
+__device__ __forceinline__ double log2p_f64_d(double a) {
+    uint64_t u = d2u(a);
+    int e = (int)((u >> 52) & 0x7FFu) - 1023;
+    double m = u2d((u & 0x000FFFFFFFFFFFFFull) | 0x3FF0000000000000ull);
+    if (m > u2d(0x3FF6A09E667F3BCDull)) { m = m * 0.5; e = e + 1; }
+    double t = (m - 1.0) / (m + 1.0);
+    double t2 = t * t;
+    double p = u2d(0x3FC1964EC6FC9491ull);
+    p = p * t2; p = p + u2d(0x3FC3703C1F4D0FFEull);
+    p = p * t2; p = p + u2d(0x3FC5B9AC9B743F0Dull);
+    p = p * t2; p = p + u2d(0x3FC89F3B1694CFFEull);
+    p = p * t2; p = p + u2d(0x3FCC68F568D31760ull);
+    p = p * t2; p = p + u2d(0x3FD0C9A84994022Dull);
+    p = p * t2; p = p + u2d(0x3FD484B13D7C02A9ull);
+    p = p * t2; p = p + u2d(0x3FDA61762A7ADED9ull);
+    p = p * t2; p = p + u2d(0x3FE2776C50EF9BFEull);
+    p = p * t2; p = p + u2d(0x3FEEC709DC3A03FDull);
+    p = p * t2; p = p + u2d(0x40071547652B82FEull);
+    double r = t * p;
+    return i2d_small(e) + r;
+}
+__device__ __forceinline__ double pow2p_f64_d(double y) {
+    const double tk = y + 6755399441055744.0;
+    double k = tk - 6755399441055744.0;
+    double f = y - k;
+    double p = u2d(0x3D7816193166D0F9ull);
+    p = p * f; p = p + u2d(0x3DBC3BD650FC2986ull);
+    p = p * f; p = p + u2d(0x3DFE8CAC7351BB25ull);
+    p = p * f; p = p + u2d(0x3E3E4CF5158B8ECAull);
+    p = p * f; p = p + u2d(0x3E7B5253D395E7C4ull);
+    p = p * f; p = p + u2d(0x3EB62C0223A5C824ull);
+    p = p * f; p = p + u2d(0x3EEFFCBFC588B0C7ull);
+    p = p * f; p = p + u2d(0x3F2430912F86C787ull);
+    p = p * f; p = p + u2d(0x3F55D87FE78A6731ull);
+    p = p * f; p = p + u2d(0x3F83B2AB6FBA4E77ull);
+    p = p * f; p = p + u2d(0x3FAC6B08D704A0C0ull);
+    p = p * f; p = p + u2d(0x3FCEBFBDFF82C58Full);
+    p = p * f; p = p + u2d(0x3FE62E42FEFA39EFull);
+    p = p * f; p = p + 1.0;
+    if (!(k <= 1023.0)) return u2d(0x7FF0000000000000ull);
+    if (k < -1022.0) return 0.0;
+    const long long ki = (long long)(d2u(tk) - 0x4338000000000000ull);
+    return p * u2d((uint64_t)(ki + 1023) << 52);
+}
+
 // predicated select that the compiler cannot turn into a branch
 __device__ __forceinline__ uint32_t selp_u32(uint32_t a, uint32_t b, bool p) {
     uint32_t r;
@@ -212,16 +299,19 @@ template <> struct QF<float> {
         uint32_t q0 = au > 0x7F800000u ? au : u;
         if (au >= 0x00800000u && au < 0x7F800000u) {
             float av = u2f(au);
-            float L = log2p_f32(av);
+            float L = log2p_f32_d(av);
             float s = L * c;
-            float rb = rintf(s);
+            // rb = rint(s) whenever |s| < 2^22; otherwise |rb| >= 2^21 and the value
+            // is stored losslessly, as with rint
+            const float ts = s + 12582912.0f;
+            float rb = ts - 12582912.0f;
             if (fabsf(rb) < 2097152.0f) {
                 float y = rb * b;
-                float r = pow2p_f32(y);
+                float r = pow2p_f32_d(y);
                 float lo = u2f(f2u(av / a) + 1u);
                 float hi = u2f(f2u(av * a) - 1u);
                 if (lo <= r && r <= hi)
-                    q0 = 0xFF800000u | (1u + ((zz(__float2int_rz(rb)) << 1) | sign));
+                    q0 = 0xFF800000u | (1u + ((zz((int32_t)(f2u(ts) - 0x4B400000u)) << 1) | sign));
             }
         }
         return q0 ^ 0xFF800000u;
@@ -230,7 +320,7 @@ template <> struct QF<float> {
         uint32_t u = w ^ 0xFF800000u;
         if ((u & 0xFF800000u) == 0xFF800000u && (u & 0x007FFFFFu) != 0) {
             uint32_t t = (u & 0x007FFFFFu) - 1u;
-            float mag = pow2p_f32(__int2float_rn(unzz(t >> 1)) * b);
+            float mag = pow2p_f32_d(i2f_small(unzz(t >> 1)) * b);     // |bin| < 2^21 (R10)
             return (t & 1u) ? -mag : mag;
         }
         return u2f(u);
@@ -261,16 +351,17 @@ template <> struct QF<double> {
         uint64_t q0 = au > 0x7FF0000000000000ull ? au : u;
         if (au >= 0x0010000000000000ull && au < 0x7FF0000000000000ull) {
             double av = u2d(au);
-            double L = log2p_f64(av);
+            double L = log2p_f64_d(av);
             double s = L * c;
-            double rb = rint(s);
+            const double ts = s + 6755399441055744.0;     // rint(s) for |s| < 2^51 (see f32)
+            double rb = ts - 6755399441055744.0;
             if (fabs(rb) < 1125899906842624.0) {
                 double y = rb * b;
-                double r = pow2p_f64(y);
+                double r = pow2p_f64_d(y);
                 double lo = u2d(d2u(av / a) + 1u);
                 double hi = u2d(d2u(av * a) - 1u);
                 if (lo <= r && r <= hi)
-                    q0 = 0xFFF0000000000000ull | (1ull + ((zz((int64_t)__double2ll_rz(rb)) << 1) | sign));
+                    q0 = 0xFFF0000000000000ull | (1ull + ((zz((int64_t)(d2u(ts) - 0x4338000000000000ull)) << 1) | sign));
             }
         }
         return q0 ^ 0xFFF0000000000000ull;
@@ -280,7 +371,7 @@ template <> struct QF<double> {
         if ((u & 0xFFF0000000000000ull) == 0xFFF0000000000000ull &&
             (u & 0x000FFFFFFFFFFFFFull) != 0) {
             uint64_t t = (u & 0x000FFFFFFFFFFFFFull) - 1u;
-            double mag = pow2p_f64(__ll2double_rn((long long)unzz(t >> 1)) * b);
+            double mag = pow2p_f64_d(i2d_small((long long)unzz(t >> 1)) * b);   // |bin| < 2^50 (R10)
             return (t & 1u) ? -mag : mag;
         }
         return u2d(u);

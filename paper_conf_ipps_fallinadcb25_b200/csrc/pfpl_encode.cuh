@@ -49,11 +49,17 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #ifndef PFPL_ENC_NQ
 #define PFPL_ENC_NQ 8
 #endif
+#ifndef PFPL_DENSE
+#define PFPL_DENSE 0
+#endif
 #ifndef PFPL_QSMEM
 #define PFPL_QSMEM 0
 #endif
 #ifndef PFPL_TIER4
 #define PFPL_TIER4 0        // P <= 4 uses the 8-plane tier: less hot code (+7% NYX)
+#endif
+#ifndef PFPL_LB_WIDE
+#define PFPL_LB_WIDE 1        // wider windows measured slower (more L2 loads): profiles/r01_tuning.md
 #endif
 #ifndef PFPL_LB_NS
 #define PFPL_LB_NS 1500
@@ -250,6 +256,26 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
         const uint32_t H = nzmark(w);
         const uint32_t o = __shfl_sync(PFPL_FULL, j < KL ? offl : offh, b & 31) +
                            __byte_perm(ex[j / 4], 0, 0x4440 + (j % 4));
+#if PFPL_DENSE
+        if (__all_sync(PFPL_FULL, H == 0x80808080u)) {
+            // dense plane (every byte of the warp's segment non-zero): the segment is the
+            // 128 bytes w_0 .. w_31 at z1 + o_0.  Aligned words 1..31 of it combine two
+            // neighbours' words (one funnel shift, one 32-bit store); the partial words at
+            // both ends are written with byte stores so no byte outside the segment is touched.
+            uint8_t* const base = z1 + (o - 4u * (uint32_t)lane);          // o_0
+            const uint32_t mis = (uint32_t)smem_u32(base) & 3u;
+            const uint32_t wprev = __shfl_up_sync(PFPL_FULL, w, 1);
+            if (lane > 0)
+                *(uint32_t*)(base - mis + 4 * lane) = __funnelshift_rc(wprev, w, 8u * (4u - mis));
+            // lanes 0..3-mis: head bytes of w_0; lanes 4..3+mis: tail bytes of w_31
+            const uint32_t we = __shfl_sync(PFPL_FULL, w, lane < 4 ? 0 : 31);
+            if ((uint32_t)lane < 4u - mis) base[lane] = (uint8_t)(we >> (8 * lane));
+            else if (lane >= 4 && (uint32_t)lane < 4u + mis)
+                base[128 - mis + (lane - 4)] = (uint8_t)(we >> (8 * (4 - mis + (lane - 4))));
+            if (!(lane & 1)) m1[pl * (CW / 64) + (tid >> 1)] = 0xFFu;
+            continue;
+        }
+#endif
         scatter_marked(z1, o, w, H);
         const uint32_t nb = nib(H >> 7);
         const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
@@ -336,23 +362,38 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             // ---- decoupled look-back ----
             uint64_t excl = 0;
             if (c > 0) {
-                // windows of 32 predecessors, lane l reads chunk look-l; the window is
-                // re-read (after a short sleep, so polling costs the compute warps
-                // almost no issue slots) until every chunk up to the first inclusive
-                // prefix has published
+                // windows of 32*LBW predecessors, lane l reads chunks look-LBW*l-j
+                // (j < LBW, nearest first).  Chunks handed out in the same "round" are
+                // processed concurrently by the other CTAs' IO warps, so the nearest
+                // inclusive prefix is typically one round (~#CTAs chunks) back: wide
+                // windows walk it in a few load latencies.  A window is re-read (after
+                // a short sleep, so polling costs the compute warps almost no issue
+                // slots) until every chunk up to the first inclusive prefix has published.
+                constexpr int LBW = PFPL_LB_WIDE;
                 int64_t look = (int64_t)c - 1;
                 const uint64_t t0 = globaltimer();
                 for (;;) {
-                    const int64_t idx = look - lane;
-                    uint64_t val = 0;
-                    uint32_t flag = (uint32_t)LB_P;               // before chunk 0: prefix 0
-                    if (idx >= 0) {
-                        const uint64_t d = ld_relaxed(&p.status[idx]);
-                        flag = ((uint32_t)(d >> 48) == p.epoch) ? (uint32_t)((d >> 46) & 3u) : 0u;
-                        val = d & LB_VAL;
+                    uint64_t d[LBW];
+                    const int64_t idx0 = look - LBW * lane;
+#pragma unroll
+                    for (int j = 0; j < LBW; ++j) d[j] = idx0 - j >= 0 ? ld_relaxed(&p.status[idx0 - j]) : 0ull;
+                    int jp = LBW;                 // nearest inclusive prefix in this lane
+                    bool nrl = false;             // a not-yet-published chunk before it
+                    uint64_t sl = 0;
+#pragma unroll
+                    for (int j = LBW - 1; j >= 0; --j) {
+                        uint32_t flag;
+                        uint64_t val;
+                        if (idx0 - j < 0) { flag = (uint32_t)LB_P; val = 0; }        // before chunk 0: prefix 0
+                        else {
+                            flag = ((uint32_t)(d[j] >> 48) == p.epoch) ? (uint32_t)((d[j] >> 46) & 3u) : 0u;
+                            val = d[j] & LB_VAL;
+                        }
+                        if (flag == LB_P) { jp = j; sl = val; nrl = false; }
+                        else { sl += val; nrl = nrl || flag == 0u; }
                     }
-                    const uint32_t pm = __ballot_sync(PFPL_FULL, flag == LB_P);
-                    const uint32_t nr = __ballot_sync(PFPL_FULL, flag == 0u);
+                    const uint32_t pm = __ballot_sync(PFPL_FULL, jp < LBW);
+                    const uint32_t nr = __ballot_sync(PFPL_FULL, nrl);
                     const uint32_t need = pm ? ((pm & (0u - pm)) << 1) - 1u : PFPL_FULL;
                     if (nr & need) {
                         // a predecessor is still being encoded (typically ~1 chunk time):
@@ -363,11 +404,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     }
                     if (pm) {
                         const int first = __ffs(pm) - 1;
-                        excl += warp_sum64(lane <= first ? val : 0ull);
+                        excl += warp_sum64(lane <= first ? sl : 0ull);
                         break;
                     }
-                    excl += warp_sum64(val);
-                    look -= 32;
+                    excl += warp_sum64(sl);
+                    look -= 32 * LBW;
                 }
                 if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + stored));
             }

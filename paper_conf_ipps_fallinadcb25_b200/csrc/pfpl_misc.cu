@@ -7,14 +7,6 @@ namespace pfpl {
 
 constexpr int MM_THREADS = 256;
 
-__device__ __forceinline__ void mm_acc(double v, double& mn, double& mx) {
-    if (isfinite(v)) {                 // R2: finite values only
-        if (v == 0.0) v = 0.0;         // canonical +0
-        mn = v < mn ? v : mn;
-        mx = v > mx ? v : mx;
-    }
-}
-
 __device__ __forceinline__ void block_minmax(double& mn, double& mx, double* out2) {
     __shared__ double smn[MM_THREADS / 32], smx[MM_THREADS / 32];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -36,22 +28,63 @@ __device__ __forceinline__ void block_minmax(double& mn, double& mx, double* out
     }
 }
 
-template <typename T>
-__global__ void __launch_bounds__(MM_THREADS) minmax_kernel(const T* in, uint64_t n, double* partial) {
-    double mn = u2d(0x7FF0000000000000ull), mx = -mn;
+// Native-precision accumulation (a T value converts to double exactly, and min/max
+// commute with that conversion): per element two FMNMX and one FSETP that records
+// whether any non-finite value was seen.  Only a thread that saw one re-reads its
+// elements with the finite filter (R2).  Zeros are canonicalised at the end (-0 and +0
+// compare equal, so which one survives the reduction never matters).
+template <typename T, bool CAREFUL>
+__device__ __forceinline__ void mm_t(T x, T& mn, T& mx, bool& nf) {
+    if (CAREFUL) {
+        if (isfinite(x)) { mn = x < mn ? x : mn; mx = x > mx ? x : mx; }
+    } else {
+        mn = fmin(mn, x);
+        mx = fmax(mx, x);
+        nf = nf || !(fabs(x) < (T)INFINITY);
+    }
+}
+template <typename T, bool CAREFUL>
+__device__ __forceinline__ void mm_pass(const T* in, uint64_t n, T& mn, T& mx, bool& nf) {
     constexpr int V = 16 / sizeof(T);
     const uint64_t nv = n / V;
     const uint64_t stride = (uint64_t)gridDim.x * MM_THREADS;
-    for (uint64_t i = (uint64_t)blockIdx.x * MM_THREADS + threadIdx.x; i < nv; i += stride) {
+    uint64_t i = (uint64_t)blockIdx.x * MM_THREADS + threadIdx.x;
+    for (; i + 3 * stride < nv; i += 4 * stride) {      // 4 loads in flight per thread
+        uint4 v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) v[u] = ldg_nc_v4(in + (i + u * stride) * V);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            T x[V];
+            memcpy(x, &v[u], 16);
+#pragma unroll
+            for (int k = 0; k < V; ++k) mm_t<T, CAREFUL>(x[k], mn, mx, nf);
+        }
+    }
+    for (; i < nv; i += stride) {
         const uint4 v = ldg_nc_v4(in + i * V);
         T x[V];
         memcpy(x, &v, 16);
 #pragma unroll
-        for (int k = 0; k < V; ++k) mm_acc((double)x[k], mn, mx);
+        for (int k = 0; k < V; ++k) mm_t<T, CAREFUL>(x[k], mn, mx, nf);
     }
-    for (uint64_t i = nv * V + (uint64_t)blockIdx.x * MM_THREADS + threadIdx.x; i < n; i += stride)
-        mm_acc((double)in[i], mn, mx);
-    block_minmax(mn, mx, partial + 2 * blockIdx.x);
+    for (uint64_t j = nv * V + (uint64_t)blockIdx.x * MM_THREADS + threadIdx.x; j < n; j += stride)
+        mm_t<T, CAREFUL>(in[j], mn, mx, nf);
+}
+template <typename T>
+__global__ void __launch_bounds__(MM_THREADS) minmax_kernel(const T* in, uint64_t n, double* partial) {
+    T mn = (T)INFINITY, mx = -(T)INFINITY;
+    bool nf = false;
+    mm_pass<T, false>(in, n, mn, mx, nf);
+    if (nf) {                                   // rare: inf/NaN among this thread's values
+        mn = (T)INFINITY;
+        mx = -(T)INFINITY;
+        mm_pass<T, true>(in, n, mn, mx, nf);
+    }
+    double dmn = (double)mn, dmx = (double)mx;
+    if (dmn == 0.0) dmn = 0.0;                  // canonical +0 (R2)
+    if (dmx == 0.0) dmx = 0.0;
+    block_minmax(dmn, dmx, partial + 2 * blockIdx.x);
 }
 
 __global__ void __launch_bounds__(MM_THREADS) minmax_final_kernel(const double* partial, int blocks,
@@ -132,7 +165,9 @@ __global__ void header_only_kernel(uint8_t* out, uint64_t n, int dtype, int boun
 // in the payload area; offs[C] = total.  Sizes are validated against the raw
 // chunk size; the total must equal the payload bytes (else *err = CORRUPT).
 // ---------------------------------------------------------------------------
-constexpr int SCAN_T = 256, SCAN_PER = 32, SCAN_TILE = SCAN_T * SCAN_PER;
+// 1024-entry tiles (NYX: 32 CTAs instead of 4), each thread 8 consecutive sizes read
+// with two 16-byte loads and written as four 16-byte stores
+constexpr int SCAN_T = 128, SCAN_PER = 8, SCAN_TILE = SCAN_T * SCAN_PER;
 
 __global__ void __launch_bounds__(SCAN_T) size_scan_kernel(const uint32_t* table, uint64_t C,
                                                             uint64_t n, uint32_t cw, uint32_t s_bytes,
@@ -149,14 +184,22 @@ __global__ void __launch_bounds__(SCAN_T) size_scan_kernel(const uint32_t* table
     const uint64_t t = sh_tile;
     const uint64_t c0 = t * SCAN_TILE + (uint64_t)tid * SCAN_PER;
     uint64_t v[SCAN_PER];
+    uint32_t szs[SCAN_PER];
     uint64_t sum = 0;
     bool bad = false;
+    if (c0 + SCAN_PER <= C) {
+        const uint4 a = *(const uint4*)(table + c0), b = *(const uint4*)(table + c0 + 4);
+        szs[0] = a.x; szs[1] = a.y; szs[2] = a.z; szs[3] = a.w;
+        szs[4] = b.x; szs[5] = b.y; szs[6] = b.z; szs[7] = b.w;
+    } else {
+#pragma unroll
+        for (int i = 0; i < SCAN_PER; ++i) szs[i] = c0 + i < C ? table[c0 + i] : 0u;
+    }
 #pragma unroll
     for (int i = 0; i < SCAN_PER; ++i) {
         const uint64_t c = c0 + i;
-        uint64_t sz = 0;
+        const uint64_t sz = szs[i];
         if (c < C) {
-            sz = table[c];
             const uint64_t m = c + 1 < C ? cw : n - c * cw;
             if (sz > m * s_bytes || (sz < 4 && sz != m * s_bytes)) bad = true;
         }
@@ -203,12 +246,22 @@ __global__ void __launch_bounds__(SCAN_T) size_scan_kernel(const uint32_t* table
     }
     __syncthreads();
     const uint64_t base = sh_excl + before + inc - sum;
+    if (c0 + SCAN_PER <= C) {
+#pragma unroll
+        for (int i = 0; i < SCAN_PER; i += 2)
+            *(ulonglong2*)(offs + c0 + i) = make_ulonglong2(base + v[i], base + v[i + 1]);
+    } else {
+#pragma unroll
+        for (int i = 0; i < SCAN_PER; ++i)
+            if (c0 + i < C) offs[c0 + i] = base + v[i];
+    }
 #pragma unroll
     for (int i = 0; i < SCAN_PER; ++i) {
         const uint64_t c = c0 + i;
-        if (c < C) offs[c] = base + v[i];
-        if (c == C - 1 && base + v[i] + table[c] != in_bytes) bad = true;
-        if (c == C - 1) offs[C] = base + v[i] + table[c];
+        if (c == C - 1) {
+            if (base + v[i] + szs[i] != in_bytes) bad = true;
+            offs[C] = base + v[i] + szs[i];
+        }
     }
     if (bad) atomicExch(err, -4);
 }
