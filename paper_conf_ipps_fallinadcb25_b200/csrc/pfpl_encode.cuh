@@ -49,9 +49,6 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #ifndef PFPL_ENC_NQ
 #define PFPL_ENC_NQ 8
 #endif
-#ifndef PFPL_DENSE
-#define PFPL_DENSE 0
-#endif
 #ifndef PFPL_QSMEM
 #define PFPL_QSMEM 0
 #endif
@@ -256,26 +253,6 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
         const uint32_t H = nzmark(w);
         const uint32_t o = __shfl_sync(PFPL_FULL, j < KL ? offl : offh, b & 31) +
                            __byte_perm(ex[j / 4], 0, 0x4440 + (j % 4));
-#if PFPL_DENSE
-        if (__all_sync(PFPL_FULL, H == 0x80808080u)) {
-            // dense plane (every byte of the warp's segment non-zero): the segment is the
-            // 128 bytes w_0 .. w_31 at z1 + o_0.  Aligned words 1..31 of it combine two
-            // neighbours' words (one funnel shift, one 32-bit store); the partial words at
-            // both ends are written with byte stores so no byte outside the segment is touched.
-            uint8_t* const base = z1 + (o - 4u * (uint32_t)lane);          // o_0
-            const uint32_t mis = (uint32_t)smem_u32(base) & 3u;
-            const uint32_t wprev = __shfl_up_sync(PFPL_FULL, w, 1);
-            if (lane > 0)
-                *(uint32_t*)(base - mis + 4 * lane) = __funnelshift_rc(wprev, w, 8u * (4u - mis));
-            // lanes 0..3-mis: head bytes of w_0; lanes 4..3+mis: tail bytes of w_31
-            const uint32_t we = __shfl_sync(PFPL_FULL, w, lane < 4 ? 0 : 31);
-            if ((uint32_t)lane < 4u - mis) base[lane] = (uint8_t)(we >> (8 * lane));
-            else if (lane >= 4 && (uint32_t)lane < 4u + mis)
-                base[128 - mis + (lane - 4)] = (uint8_t)(we >> (8 * (4 - mis + (lane - 4))));
-            if (!(lane & 1)) m1[pl * (CW / 64) + (tid >> 1)] = 0xFFu;
-            continue;
-        }
-#endif
         scatter_marked(z1, o, w, H);
         const uint32_t nb = nib(H >> 7);
         const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
