@@ -140,6 +140,43 @@ int pfpl_last_cuda_error(void);
 int pfpl_watchdog_report(unsigned int* out4);
 /* Frees the calling thread's scratch for the current device. */
 int pfpl_release_scratch(void);
+/* Reconstruction-quality metrics of a decompression against the original values
+ * (the paper's Fig. 16 analogue), accumulated in the
+ * decoder's epilogue in f64 arithmetic (exact differences for f32 data).  Finite
+ * originals only, except `violations`, which also counts non-finite originals that
+ * did not come back bit-identical (REL: NaN sign cleared). */
+typedef struct {
+    uint64_t n;             /* values decoded */
+    uint64_t n_finite;      /* finite original values */
+    double max_abs_err;     /* max |x - y| */
+    double max_rel_err;     /* max |x - y| / |x| over x != 0 */
+    double sum_sq_err;      /* sum (x - y)^2 (summation order is unspecified) */
+    double mse;             /* sum_sq_err / n_finite */
+    double psnr;            /* 20 log10(value_max - value_min) - 10 log10(mse); +inf if mse == 0 */
+    double value_min, value_max;   /* range of the finite originals */
+    uint64_t violations;    /* values outside the stream's bound (ABS eps, REL eps*|x|,
+                               NOA eps*range) -- must be 0 */
+} pfpl_metrics;
+
+/* pfpl_decompress plus verification: `orig` (device, 16-byte aligned, n values of the
+ * stream's dtype, as given to pfpl_compress) is read once, alongside the decode, and
+ * *m is filled on return.  Same arguments, ownership, sync and errors as
+ * pfpl_decompress; PFPL_ERR_ARG if orig or m is null, PFPL_ERR_ALIGN if orig is
+ * misaligned.  Costs one extra read of n values. */
+int pfpl_decompress_verify(const void* in, uint64_t in_bytes, const void* orig, void* out,
+                           uint64_t* out_bytes, pfpl_metrics* m, void* stream);
+
+/* Statistics of the most recent compression enqueued on `stream` (current
+ * device), counted inside the encoder at no cost on chunks without them:
+ *   *unquantizable = values whose bin failed the reconstruct-and-verify check
+ *                    (or all values in raw-words mode) and were stored
+ *                    losslessly -- the paper's "unquantizable values";
+ *   *raw_chunks    = chunks stored as raw bytes because the encoded chunk was not
+ *                    smaller.
+ * Synchronizes `stream`.  Zeros if nothing was compressed on it yet.  A later
+ * compression on the same stream overwrites them.  Returns PFPL_OK,
+ * PFPL_ERR_ARG (null output) or PFPL_ERR_CUDA. */
+int pfpl_last_stats(void* stream, uint64_t* unquantizable, uint64_t* raw_chunks);
 /* Number of kernel launches issued by the library since load (for bench's
  * gpu_launches claim). */
 uint64_t pfpl_launch_count(void);

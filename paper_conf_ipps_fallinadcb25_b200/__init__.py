@@ -66,6 +66,8 @@ def lib():
             "pfpl_watchdog_report": (i32, [ctypes.POINTER(ctypes.c_uint)]),
             "pfpl_release_scratch": (i32, []),
             "pfpl_launch_count": (u64, []),
+            "pfpl_last_stats": (i32, [vp, pu64, pu64]),
+            "pfpl_decompress_verify": (i32, [vp, u64, vp, vp, pu64, vp, vp]),
             "pfpl_version": (ctypes.c_char_p, []),
         }
         for name, (res, args) in sig.items():
@@ -178,6 +180,38 @@ def decompress(buf: torch.Tensor, out: torch.Tensor | None = None, stream=None) 
     return out[:h["n"]]
 
 
+class Metrics(ctypes.Structure):
+    """pfpl_metrics (include/pfpl.h)"""
+    _fields_ = [("n", ctypes.c_uint64), ("n_finite", ctypes.c_uint64), ("max_abs_err", ctypes.c_double),
+                ("max_rel_err", ctypes.c_double), ("sum_sq_err", ctypes.c_double), ("mse", ctypes.c_double),
+                ("psnr", ctypes.c_double), ("value_min", ctypes.c_double), ("value_max", ctypes.c_double),
+                ("violations", ctypes.c_uint64)]
+
+
+def decompress_verify(buf: torch.Tensor, orig: torch.Tensor, out: torch.Tensor | None = None,
+                      stream=None):
+    """Decompress and measure the reconstruction against `orig` in the same pass
+    (SURVEY 8(f) NEXT-3): returns (values, metrics dict)."""
+    _require_cuda(buf, "buf")
+    _require_cuda(orig, "orig")
+    if buf.numel() < HEADER_BYTES:
+        raise PFPLError(-4, "stream shorter than its header")
+    hdr = buf[:HEADER_BYTES].cpu().numpy().tobytes()
+    h = peek_header(hdr)
+    tdt = torch.float32 if h["dtype"] == F32 else torch.float64
+    if orig.dtype != tdt or orig.numel() != h["n"] or not orig.is_contiguous():
+        raise PFPLError(-1, "orig must be a contiguous tensor of the stream's dtype and length")
+    if out is None:
+        out = torch.empty(max(h["n"], 1), dtype=tdt, device=buf.device)
+    ob = ctypes.c_uint64(out.numel() * out.element_size())
+    m = Metrics()
+    with torch.cuda.device(buf.device):
+        st = lib().pfpl_decompress_verify(buf.data_ptr(), buf.numel(), orig.data_ptr(), out.data_ptr(),
+                                          ctypes.byref(ob), ctypes.byref(m), _stream(stream))
+    _check(st, "decompress_verify")
+    return out[:h["n"]], {k: getattr(m, k) for k, _ in Metrics._fields_}
+
+
 def decompress_async(buf: torch.Tensor, hdr: bytes, out: torch.Tensor, result: torch.Tensor,
                      stream=None) -> None:
     h = ctypes.create_string_buffer(bytes(hdr[:HEADER_BYTES]), HEADER_BYTES)
@@ -230,6 +264,16 @@ def decompress_chunks(hdr: bytes, table, first_chunk: int, payload: torch.Tensor
                                       payload.numel(), out.data_ptr(),
                                       out.numel() * out.element_size(), _stream(stream))
     _check(st, "decompress_chunks")
+
+
+def last_stats(stream=None) -> dict:
+    """Counters of the most recent compression on `stream` (default: the current
+    stream): unquantizable values stored losslessly and raw chunks."""
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    u, r = ctypes.c_uint64(0), ctypes.c_uint64(0)
+    _check(lib().pfpl_last_stats(s.cuda_stream, ctypes.byref(u), ctypes.byref(r)))
+    return {"unquantizable": u.value, "raw_chunks": r.value}
 
 
 def launch_count() -> int:

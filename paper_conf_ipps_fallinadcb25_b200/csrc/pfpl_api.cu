@@ -39,6 +39,9 @@ struct Scratch {
     uint64_t table_cap = 0;
     uint64_t* offs = nullptr;        // decoder chunk offsets (C + 1)
     uint64_t offs_cap = 0;
+    unsigned long long* stats = nullptr;   // 2 slots x {unquantizable values, raw chunks}
+    unsigned long long* vm = nullptr;      // verify-mode metric accumulators (8)
+    uint64_t stat_seq = 0;                 // compress calls enqueued (slot = seq & 1)
 };
 
 std::mutex g_mu;
@@ -82,6 +85,8 @@ int get_scratch(cudaStream_t s, uint64_t C, Scratch** out) {
         CK(cudaMalloc(&sc->result, 4 * sizeof(uint64_t)));
         CK(cudaMallocHost(&sc->host, 4 * sizeof(uint64_t)));
         CK(cudaMallocHost(&sc->hdr_host, 64));
+        CK(cudaMalloc(&sc->stats, 4 * sizeof(unsigned long long)));
+        CK(cudaMemsetAsync(sc->stats, 0, 4 * sizeof(unsigned long long), s));
     }
     if (C > sc->status_cap) {
         if (sc->status) CK(cudaFreeAsync(sc->status, s));
@@ -207,7 +212,13 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
         g_launches += 1;
         qdev = sc->qc_dev;
     }
+    // statistics slot of this call; the kernel zeroes the other slot for the next one
+    unsigned long long* const st_cur = sc->stats + 2 * (sc->stat_seq & 1);
+    unsigned long long* const st_next = sc->stats + 2 * ((sc->stat_seq + 1) & 1);
+    sc->stat_seq += 1;
     if (C == 0) {
+        // no kernel runs to zero the next slot: clear both
+        CK(cudaMemsetAsync(sc->stats, 0, 4 * sizeof(unsigned long long), s));
         if (write_header) {
             CK(launch_header_only(out, n_total, dtype, bound, eps, qc, qdev, result, s));
         } else {
@@ -242,6 +253,8 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
     p.dtype = (uint32_t)dtype;
     p.bound = (uint32_t)bound;
     p.wd = watchdog_ptr();
+    p.stats = st_cur;
+    p.stats_next = st_next;
     const bool ms = (opts & PFPL_OPT_MS_RESIDUALS) != 0;
     const int grid = encode_grid(dtype, mode, ms, C);
     CK(launch_encode(dtype, mode, ms, p, grid, s));
@@ -307,11 +320,13 @@ int decode_qconst(int dtype, int bound, unsigned flags, uint64_t qk, QConst* qc,
 
 int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t first_chunk,
                        uint64_t nchunks, const uint8_t* payload, uint64_t payload_bytes,
-                       void* out, uint64_t cap, int* err_dev, cudaStream_t s, uint64_t* n_out) {
+                       void* out, uint64_t cap, int* err_dev, cudaStream_t s, uint64_t* n_out,
+                       const void* orig = nullptr, unsigned long long* vm = nullptr) {
     uint64_t n = 0, qk = 0;
     int dtype = 0, bound = 0;
     unsigned flags = 0;
-    int st = parse_header(hdr, kHeaderBytes, &n, &dtype, &bound, nullptr, &flags, &qk, nullptr);
+    double eps_h = 0.0, range_h = 0.0;
+    int st = parse_header(hdr, kHeaderBytes, &n, &dtype, &bound, &eps_h, &flags, &qk, &range_h);
     if (st != PFPL_OK) return st;
     QConst qc;
     int mode = 0;
@@ -356,6 +371,11 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     p.err = err_dev;
     p.wd = watchdog_ptr();
     p.c23 = dtype == PFPL_F32 ? f2u_h(u2f_h((uint32_t)qc.c) * 8388608.0f) : 0u;   // exact or inf
+    p.orig = orig;
+    p.vm = vm;
+    p.vbound = bound;
+    p.veps = eps_h;
+    p.vrange = range_h;
     const bool ms = (flags & HF_MS) != 0;
     const int grid = decode_grid(dtype, mode, ms, nchunks);
     CK(launch_decode(dtype, mode, ms, p, grid, s));
@@ -470,6 +490,61 @@ int pfpl_decompress(const void* in, uint64_t in_bytes, void* out, uint64_t* out_
     const int err = (int)(int32_t)(uint32_t)sc->host[1];
     if (err) return err;
     *out_bytes = nout * tsz(dtype);
+    return PFPL_OK;
+}
+
+int pfpl_decompress_verify(const void* in, uint64_t in_bytes, const void* orig, void* out,
+                           uint64_t* out_bytes, pfpl_metrics* m, void* stream) {
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!in || !out_bytes || !orig || !m) return PFPL_ERR_ARG;
+    if (!aligned16(in) || !aligned16(orig)) return PFPL_ERR_ALIGN;
+    if (in_bytes < kHeaderBytes) return PFPL_ERR_CORRUPT;
+    memset(m, 0, sizeof(*m));
+    Scratch* sc = nullptr;
+    int st = get_scratch(s, 0, &sc);
+    if (st != PFPL_OK) return st;
+    if (!sc->vm) CK(cudaMalloc(&sc->vm, 8 * sizeof(unsigned long long)));
+    CK(cudaMemcpyAsync(sc->hdr_host, in, kHeaderBytes, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    uint8_t hdr[kHeaderBytes];
+    memcpy(hdr, sc->hdr_host, kHeaderBytes);
+    uint64_t n = 0;
+    int dtype = 0, bound = 0;
+    double eps = 0.0, range = 0.0;
+    st = parse_header(hdr, kHeaderBytes, &n, &dtype, &bound, &eps, nullptr, nullptr, &range);
+    if (st != PFPL_OK) return st;
+    const uint64_t C = chunks_of(n, dtype);
+    if (in_bytes < kHeaderBytes + 4 * C) return PFPL_ERR_CORRUPT;
+    // accumulators: zeros, min = order(+inf), max = order(-inf)
+    static const unsigned long long init[8] = {0, 0, 0, 0, 0, 0xFFF0000000000000ull /* ord(+inf) */,
+                                               ~0xFFF0000000000000ull /* ord(-inf) */, 0};
+    CK(cudaMemcpyAsync(sc->vm, init, sizeof(init), cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(sc->result + 1, 0, 8, s));
+    const uint8_t* base = (const uint8_t*)in;
+    uint64_t nout = 0;
+    st = enqueue_decompress(hdr, (const uint32_t*)(base + kHeaderBytes), 0, C,
+                            base + kHeaderBytes + 4 * C, in_bytes - kHeaderBytes - 4 * C, out,
+                            *out_bytes, (int*)(sc->result + 1), s, &nout, orig, sc->vm);
+    if (st != PFPL_OK) return st;
+    unsigned long long v[8];
+    CK(cudaMemcpyAsync(sc->host + 1, sc->result + 1, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(v, sc->vm, sizeof(v), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    const int err = (int)(int32_t)(uint32_t)sc->host[1];
+    if (err) return err;
+    *out_bytes = nout * tsz(dtype);
+    auto unord = [](unsigned long long o) { return u2d_h((o >> 63) ? (o & 0x7FFFFFFFFFFFFFFFull) : ~o); };
+    m->n = n;
+    m->n_finite = v[4];
+    m->max_abs_err = u2d_h(v[0]);
+    m->max_rel_err = u2d_h(v[1]);
+    m->sum_sq_err = u2d_h(v[2]);
+    m->violations = v[3];
+    m->value_min = v[4] ? unord(v[5]) : 0.0;
+    m->value_max = v[4] ? unord(v[6]) : 0.0;
+    m->mse = v[4] ? m->sum_sq_err / (double)v[4] : 0.0;
+    const double rng = m->value_max - m->value_min;
+    m->psnr = (m->mse > 0.0 && rng > 0.0) ? 20.0 * log10(rng) - 10.0 * log10(m->mse) : INFINITY;
     return PFPL_OK;
 }
 
@@ -588,9 +663,32 @@ int pfpl_release_scratch(void) {
         cudaFree(sc->status); cudaFree(sc->ticket); cudaFree(sc->qc_dev); cudaFree(sc->mnmx);
         cudaFree(sc->partial); cudaFree(sc->result); cudaFreeHost(sc->host);
         cudaFreeHost(sc->hdr_host); cudaFree(sc->table_dev); cudaFree(sc->offs);
+        cudaFree(sc->stats); cudaFree(sc->vm);
         delete sc;
         it = g_scratch.erase(it);
     }
+    return PFPL_OK;
+}
+
+int pfpl_last_stats(void* stream, uint64_t* unquantizable, uint64_t* raw_chunks) {
+    if (!unquantizable || !raw_chunks) return PFPL_ERR_ARG;
+    *unquantizable = 0;
+    *raw_chunks = 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    Scratch* sc = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        auto it = g_scratch.find({dev, (void*)s});
+        if (it != g_scratch.end()) sc = it->second;
+    }
+    if (!sc || sc->stat_seq == 0) return PFPL_OK;          // no compression on this stream yet
+    unsigned long long v[2];
+    CK(cudaMemcpyAsync(v, sc->stats + 2 * ((sc->stat_seq - 1) & 1), sizeof(v), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    *unquantizable = v[0];
+    *raw_chunks = v[1];
     return PFPL_OK;
 }
 

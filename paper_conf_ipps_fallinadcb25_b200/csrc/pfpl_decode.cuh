@@ -20,6 +20,7 @@
 //                                              a TMA 2-D tensor store
 #pragma once
 #include <cuda.h>
+#include <type_traits>
 #include "pfpl_device.cuh"
 
 namespace pfpl {
@@ -152,7 +153,67 @@ __device__ __forceinline__ void dec1_gather(uint32_t (&lo)[32], uint32_t (&hi)[3
 
 __device__ __forceinline__ void set_err(int* err) { atomicExch(err, -4); }
 
-template <typename T, int MODE, bool MSR>
+// order-preserving map of a double to u64 (for atomicMin / atomicMax)
+__device__ __forceinline__ unsigned long long ord_u64(double v) {
+    const uint64_t u = d2u(v);
+    return (u >> 63) ? ~u : (u | 0x8000000000000000ull);
+}
+
+// Verify mode: reconstruction-quality metrics of the decoded values y
+// against the originals x, accumulated in the decode epilogue (Fig. 16), and a
+// count of values outside the stream's bound -- in f64 arithmetic, exact for f32
+// data.  Non-finite x must come back bit-identical (REL: NaN sign cleared).
+template <typename T>
+struct VerAcc {
+    double mabs = 0.0, mrel = 0.0, ssq = 0.0, vmin = INFINITY, vmax = -INFINITY;
+    unsigned long long nviol = 0, nfin = 0;
+    __device__ __forceinline__ void add(T x, T y, const DecParams& p) {
+        const double xd = (double)x, yd = (double)y;
+        if (isfinite(xd)) {
+            const double d = fabs(xd - yd);
+            mabs = fmax(mabs, d);
+            ssq += d * d;
+            if (xd != 0.0) mrel = fmax(mrel, d / fabs(xd));
+            vmin = fmin(vmin, xd);
+            vmax = fmax(vmax, xd);
+            nfin += 1;
+            const double lim = p.vbound == 1 ? p.veps * fabs(xd) : p.vbound == 2 ? p.veps * p.vrange : p.veps;
+            if (!(d <= lim)) nviol += 1;
+        } else if (!((isnan(xd) && isnan(yd)) || xd == yd)) {
+            nviol += 1;
+        }
+    }
+    __device__ __forceinline__ void flush(const DecParams& p) {
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) {
+            mabs = fmax(mabs, __shfl_xor_sync(PFPL_FULL, mabs, d));
+            mrel = fmax(mrel, __shfl_xor_sync(PFPL_FULL, mrel, d));
+            ssq += __shfl_xor_sync(PFPL_FULL, ssq, d);
+            vmin = fmin(vmin, __shfl_xor_sync(PFPL_FULL, vmin, d));
+            vmax = fmax(vmax, __shfl_xor_sync(PFPL_FULL, vmax, d));
+            nviol += __shfl_xor_sync(PFPL_FULL, nviol, d);
+            nfin += __shfl_xor_sync(PFPL_FULL, nfin, d);
+        }
+        if ((threadIdx.x & 31) == 0) {
+            atomicMax(&p.vm[0], (unsigned long long)d2u(mabs));      // non-negative: bits order
+            atomicMax(&p.vm[1], (unsigned long long)d2u(mrel));
+            atomicAdd((double*)&p.vm[2], ssq);
+            if (nviol) atomicAdd(&p.vm[3], nviol);
+            atomicAdd(&p.vm[4], nfin);
+            if (nfin) {
+                atomicMin(&p.vm[5], ord_u64(vmin));
+                atomicMax(&p.vm[6], ord_u64(vmax));
+            }
+        }
+    }
+};
+template <typename T>
+struct VerNone {
+    __device__ __forceinline__ void add(T, T, const DecParams&) {}
+    __device__ __forceinline__ void flush(const DecParams&) {}
+};
+
+template <typename T, int MODE, bool MSR, bool VER = false>
 __global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_DEC_MINB : 4)
 decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
@@ -272,6 +333,8 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     const bool raw = (p.qc.flags & HF_RAWWORDS) != 0;
     const float c23 = u2f((uint32_t)p.c23);
     const bool fastdq = sizeof(T) == 4 && MODE == MODE_ABS && !isinf(c23);
+    typename std::conditional<VER, VerAcc<T>, VerNone<T>>::type vacc;
+    const T* const orig = (const T*)p.orig;
     for (uint32_t it = 0;; ++it) {
         const int slot = it % NQD;
         mbar_wait_wd(smem_u32(&S.full[slot]), (it / NQD) & 1u, 0x22);
@@ -303,6 +366,10 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             }
             named_sync(1, NTC);
             release();
+            if constexpr (VER) {       // the chunk's words were written by the whole CTA
+                for (uint32_t e = tid; e < m; e += NTC)
+                    vacc.add(orig[c * (uint64_t)CW + e], ((const T*)dstc)[e], p);
+            }
             continue;
         }
         // ---- levels 4 -> 3 -> 2, derived by every warp (no barrier) ----
@@ -501,15 +568,35 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 tma_store_2d(&tmap, 0, (int)(c * 128), smem_u32(stage_out));
                 bulk_commit();
             }
+            if constexpr (VER) {
+                // this thread's staged rows against the originals (16-byte loads; each
+                // sector of the original chunk is read once)
+#pragma unroll 1
+                for (int i = 0; i < 2 * S_; ++i) {
+                    const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
+                    const uint4 v = *(const uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4));
+                    const uint4 o = ldg_nc_v4(orig + c * (uint64_t)CW + (uint64_t)(r * (128 / S_) + (i & 7) * (16 / S_)));
+                    T y[16 / S_], x[16 / S_];
+                    memcpy(y, &v, 16);
+                    memcpy(x, &o, 16);
+#pragma unroll
+                    for (int k = 0; k < 16 / S_; ++k) vacc.add(x[k], y[k], p);
+                }
+            }
         } else {
             // tail chunk: plain stores of the first m values
 #pragma unroll
             for (int i = 0; i < 32; ++i) {
                 const uint32_t e = 32 * tid + i;
-                if (e < m) ((T*)dstc)[e] = dequantize<T, MODE>(q, (W)(carry + dq[i]), raw);
+                if (e < m) {
+                    const T yv = dequantize<T, MODE>(q, (W)(carry + dq[i]), raw);
+                    ((T*)dstc)[e] = yv;
+                    if constexpr (VER) vacc.add(orig[c * (uint64_t)CW + e], yv, p);
+                }
             }
         }
     }
+    if constexpr (VER) vacc.flush(p);
     if (tid == 0) bulk_wait0();    // all TMA stores of this CTA complete before exit
 }
 

@@ -49,6 +49,9 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #ifndef PFPL_ENC_NQ
 #define PFPL_ENC_NQ 8
 #endif
+#ifndef PFPL_STATS
+#define PFPL_STATS 1
+#endif
 #ifndef PFPL_QSMEM
 #define PFPL_QSMEM 0
 #endif
@@ -276,6 +279,20 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
         }                                                                               \
     } while (0)
 
+// A word is a bin (quantized value) iff it lies in the bin range of its mode: ABS/NOA
+// zigzag bins below the normal range (R8; f32 words carry the encoder's bias), REL bins
+// 1 + payload in the (inverted) negative-NaN pattern (R10, R11).  Everything else, and
+// every word in raw-words mode, is an unquantizable value stored losslessly.
+template <typename T, int MODE>
+__device__ __forceinline__ bool is_bin_word(typename Tr<T>::W w, typename Tr<T>::W qbias, bool raw) {
+    typedef typename Tr<T>::W W;
+    constexpr W LIM = sizeof(T) == 4 ? (W)0x00800000u : (W)0x0010000000000000ull;
+    if (!PFPL_STATS) return true;
+    if (MODE == MODE_RAW || (MODE == MODE_NOA && raw)) return false;
+    if (MODE == MODE_REL) return (W)(w - 1) < (W)(LIM - 1);
+    return (W)(w - qbias) < LIM;
+}
+
 template <typename T, int MODE, bool MSR>
 __global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_ENC_MINB : 5)
 encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
@@ -308,6 +325,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     unsigned long long next = 0;
     if (tid == 0) {
         g_pfpl_wd = p.wd;
+        if (blockIdx.x == 0 && p.stats_next) { p.stats_next[0] = 0; p.stats_next[1] = 0; }
         if (smem_u32(smem) & 1023u) __trap();       // TMA SWIZZLE_128B needs 1024-byte alignment
         for (int s = 0; s < NIN; ++s) mbar_init(smem_u32(&S.full[s]), 1);
         for (int k = 0; k < NQ; ++k) {
@@ -446,6 +464,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         // ---- quantize + verify, delta, residual code ----
         uint32_t lo[32], hi[32];
         W orv = 0;
+        // unquantizable values (0 on the fast path): counted on the other paths only
+        auto add_raw = [&](uint32_t nraw) {
+            const uint32_t t = __reduce_add_sync(PFPL_FULL, nraw);
+            if (lane == 0 && t && p.stats) atomicAdd(&p.stats[0], (unsigned long long)t);
+        };
         {
             // biased words (quantize_b): q + bias; the bias cancels in q[i] - q[i-1]
             W qprev = (W)qbias;
@@ -546,6 +569,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         }
                     }
                     __syncwarp();
+                    uint32_t nraw = 0;
 #pragma unroll 1
                     for (int i = 0; i < 2 * S_; ++i) {
                         const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
@@ -555,10 +579,14 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         W w[16 / S_];
                         memcpy(x, &v, 16);
 #pragma unroll
-                        for (int k = 0; k < 16 / S_; ++k) w[k] = quantize_b<T, MODE>(q, x[k], raw);
+                        for (int k = 0; k < 16 / S_; ++k) {
+                            w[k] = quantize_b<T, MODE>(q, x[k], raw);
+                            nraw += is_bin_word<T, MODE>(w[k], (W)qbias, raw) ? 0u : 1u;
+                        }
                         memcpy(&v, w, 16);
                         *a = v;
                     }
+                    add_raw(nraw);
                     if (tid > 0) qprev = quantize_b<T, MODE>(q, pv, raw);
                     fence_proxy_async();      // the stage is refilled by TMA after the next barrier
 #pragma unroll
@@ -592,6 +620,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     }
                     qprev = quantize_b<T, MODE>(q, pv, raw);
                 }
+                uint32_t nraw = 0;
 #pragma unroll
                 for (int i = 0; i < 2 * S_; ++i) {
                     const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
@@ -601,6 +630,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
 #pragma unroll
                     for (int k = 0; k < 16 / S_; ++k) {
                         const W qw = quantize_b<T, MODE>(q, x[k], raw);
+                        nraw += is_bin_word<T, MODE>(qw, (W)qbias, raw) ? 0u : 1u;
                         const W r2 = rcode<MSR>((W)(qw - qprev));
                         qprev = qw;
                         orv |= r2;
@@ -608,20 +638,24 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         hi[i * (16 / S_) + k] = sizeof(W) == 8 ? (uint32_t)((uint64_t)r2 >> 32) : 0u;
                     }
                 }
+                add_raw(nraw);
             } else {
                 // tail chunk (or a clobbered stage): plain loads; R12 pads with the last
                 // value -> zero residuals
                 const T* src = (const T*)p.in + c * (uint64_t)CW;
                 if (tid > 0) qprev = quantize_b<T, MODE>(q, src[min(32 * tid - 1, (int)m - 1)], raw);
+                uint32_t nraw = 0;
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
                     const W qw = quantize_b<T, MODE>(q, src[min(32 * tid + i, (int)m - 1)], raw);
+                    if (32 * tid + i < (int)m) nraw += is_bin_word<T, MODE>(qw, (W)qbias, raw) ? 0u : 1u;
                     const W r2 = rcode<MSR>((W)(qw - qprev));
                     qprev = qw;
                     orv |= r2;
                     lo[i] = (uint32_t)r2;
                     hi[i] = sizeof(W) == 8 ? (uint32_t)((uint64_t)r2 >> 32) : 0u;
                 }
+                add_raw(nraw);
             }
         }
         // this warp's active planes (warp-uniform tier; other warps may differ)
@@ -748,6 +782,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const uint32_t size = 4 + n4 + n3 + n2 + n1;
             const uint32_t rawb = m * S_;
             const bool israw = size >= rawb;
+            if (israw && lane == 0 && p.stats) atomicAdd(&p.stats[1], 1ull);
             const uint32_t stored = israw ? rawb : size;
             __syncwarp();
             if (lane == 0) {

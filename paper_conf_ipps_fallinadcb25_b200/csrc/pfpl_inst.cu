@@ -20,7 +20,17 @@ typedef float InstT;
 #else
 typedef double InstT;
 #endif
+#if PFPL_KIND == 0
 void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms) {
     return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false>;
 }
+#else
+// decoder: (residual code, verify mode); verify is instantiated for the default residuals
+// and for zigzag residuals alike
+void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms, bool ver) {
+    if (ver) return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, true>
+                       : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, true>;
+    return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, false> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, false>;
+}
+#endif
 }  // namespace pfpl

@@ -45,6 +45,8 @@ struct EncParams {
     double eps;              // header eps
     uint32_t dtype, bound;   // header bytes 5, 6
     unsigned int* wd;        // watchdog report (mapped host memory) or null
+    unsigned long long* stats;       // [0] unquantizable values, [1] raw chunks (this call)
+    unsigned long long* stats_next;  // the other slot: zeroed for the next call
 };
 
 struct DecParams {
@@ -63,13 +65,20 @@ struct DecParams {
     uint64_t c23;            // f32 ABS: bits of 2^23 * eb2 (inf if it overflows)
     const uint64_t* offs;    // offs[c] = byte offset of chunk c's payload (size_scan_kernel)
     unsigned int* wd;        // watchdog report (mapped host memory) or null
+    // verify mode (pfpl_decompress_verify): original values and the metric accumulators
+    // vm[0] max |x-y| (f64 bits), [1] max |x-y|/|x| (f64 bits), [2] sum (x-y)^2 (f64),
+    // [3] bound violations, [4] finite values, [5] / [6] order-mapped min / max of x
+    const void* orig;
+    unsigned long long* vm;
+    int vbound;              // bound of the stream (header byte 6)
+    double veps, vrange;     // user eps and the NOA range d (header fields)
 };
 
 // kernel launchers (pfpl_kernels.cu)
 cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int grid,
                           cudaStream_t s);
 cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
-                          cudaStream_t s);
+                          cudaStream_t s);   // p.orig != null selects the verify kernel
 int scan_grid(uint64_t C);
 cudaError_t launch_size_scan(const uint32_t* table, uint64_t C, uint64_t n, uint32_t cw,
                              uint32_t s_bytes, uint64_t in_bytes, uint64_t* offs,

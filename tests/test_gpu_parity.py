@@ -199,3 +199,102 @@ def test_repeat_determinism(pk, name, bound, eps):
         n = int(rc[0])
         assert n == ref.numel() and torch.equal(out[:n], ref), f"rep {i}: stream differs"
         assert int(rd[1]) == 0 and torch.equal(y, y0), f"rep {i}: decode differs"
+
+
+# ---- encoder statistics (pfpl_last_stats): unquantizable values, raw chunks
+def _oracle_unquantizable(orc, x: np.ndarray, bound: str, eps: float) -> int:
+    """Values the oracle's quantizer (O1) stores losslessly: words outside the bin
+    range of the stream format (R8 ABS/NOA zigzag bins below the normal range, R10 REL
+    bins 1 + payload), or every value in raw-words mode (R4)."""
+    P = orc.params(x, bound, eps)
+    if P.flags & 1:
+        return x.size
+    w = orc.quantize(x, bound, eps, P).astype(np.uint64)
+    lim = np.uint64(2**23 if x.dtype == np.float32 else 2**52)
+    if bound == "rel":
+        return int(np.count_nonzero(~((w >= 1) & (w < lim))))
+    return int(np.count_nonzero(w >= lim))
+
+
+def _raw_chunks(stream: bytes, x: np.ndarray) -> int:
+    cw = 16384 // x.itemsize
+    C = -(-x.size // cw)
+    sizes = np.frombuffer(stream[48:48 + 4 * C], np.uint32)
+    raw = [(min(cw, x.size - c * cw) * x.itemsize) for c in range(C)]
+    return int(np.count_nonzero(sizes == np.array(raw, np.uint32)))
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_stats_match_oracle(pk, orc, dt):
+    rng = np.random.default_rng(11)
+    adv = synth.adversarial_f32() if dt == np.float32 else synth.adversarial_f64()
+    n = 3 * (16384 // np.dtype(dt).itemsize) + 5
+    u = rng.integers(0, 2**63, size=n, dtype=np.int64).astype(np.uint64)
+    rnd = (u.astype(np.uint32) if dt == np.float32 else u).view(dt)
+    spec = synth.FieldSpec("t", (20000,), "f32" if dt == np.float32 else "f64", 3, A=0.5, tau=0.01)
+    fld = synth.generate(spec).numpy()
+    fld[::97] = np.inf                      # a sprinkle of unquantizable values in a smooth field
+    cases = [(adv, b, e) for b in ("abs", "rel", "noa") for e in (1e-1, 1e-4)]
+    cases += [(rnd, b, 1e-3) for b in ("abs", "rel", "noa")]
+    cases += [(fld, b, 1e-3) for b in ("abs", "rel", "noa")]
+    cases += [(np.zeros(0, dt), "abs", 1e-3)]
+    for x, bound, eps in cases:
+        s = pk.compress(torch.from_numpy(x).cuda(), bound, eps).cpu().numpy().tobytes()
+        st = pk.last_stats()
+        want_u = _oracle_unquantizable(orc, x, bound, eps)
+        assert st["unquantizable"] == want_u, (bound, eps, x.size, st, want_u)
+        assert st["raw_chunks"] == _raw_chunks(s, x), (bound, eps, x.size, st)
+
+
+# ---- verify mode (pfpl_decompress_verify, SURVEY 8(f) NEXT-3)
+def _metrics_ref(x: np.ndarray, y: np.ndarray, bound: str, eps: float, rng_noa: float):
+    xd, yd = x.astype(np.float64), y.astype(np.float64)
+    fin = np.isfinite(xd)
+    d = np.abs(xd[fin] - yd[fin])
+    nz = xd[fin] != 0
+    lim = {"abs": np.full(d.shape, eps), "rel": eps * np.abs(xd[fin]),
+           "noa": np.full(d.shape, eps * rng_noa)}[bound]
+    nonfin_bad = ~fin & ~((np.isnan(xd) & np.isnan(yd)) | (xd == yd))
+    return dict(n_finite=int(fin.sum()), max_abs_err=float(d.max()) if d.size else 0.0,
+                max_rel_err=float((d[nz] / np.abs(xd[fin][nz])).max()) if nz.any() else 0.0,
+                sum_sq_err=float((d * d).sum()), violations=int((~(d <= lim)).sum() + nonfin_bad.sum()),
+                value_min=float(xd[fin].min()) if fin.any() else 0.0,
+                value_max=float(xd[fin].max()) if fin.any() else 0.0)
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+@pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
+def test_decompress_verify_metrics(pk, orc, dt, bound):
+    """Metrics from the decode epilogue equal numpy's on the oracle-decoded values (max
+    and counts exactly, the f64 sum up to summation order); zero violations; a perturbed
+    original is caught value by value."""
+    spec = synth.FieldSpec("t", (3 * 4096 + 1000,), "f32" if dt == np.float32 else "f64", 5, A=0.5, tau=0.01)
+    cases = [synth.generate(spec).numpy(),
+             synth.adversarial_f32() if dt == np.float32 else synth.adversarial_f64()]
+    rng = np.random.default_rng(3)
+    u = rng.integers(0, 2**63, size=2 * (16384 // np.dtype(dt).itemsize) + 7, dtype=np.int64).astype(np.uint64)
+    cases.append((u.astype(np.uint32) if dt == np.float32 else u).view(dt))     # raw chunks
+    for ci, x in enumerate(cases):
+        eps = 1e-3
+        s = orc.compress(x, bound, eps)
+        P = orc.params(x, bound, eps)
+        y_ref = orc.decompress(s)
+        buf = torch.frombuffer(bytearray(s), dtype=torch.uint8).cuda()
+        xg = torch.from_numpy(x).cuda()
+        y, m = pk.decompress_verify(buf, xg)
+        assert np.array_equal(_bits(y.cpu().numpy()), _bits(y_ref))
+        ref = _metrics_ref(x, y_ref, bound, eps, P.range)
+        assert m["n"] == x.size and m["n_finite"] == ref["n_finite"]
+        assert m["violations"] == 0 == ref["violations"]
+        assert m["max_abs_err"] == ref["max_abs_err"] and m["max_rel_err"] == ref["max_rel_err"]
+        assert m["value_min"] == ref["value_min"] and m["value_max"] == ref["value_max"]
+        assert m["sum_sq_err"] == pytest.approx(ref["sum_sq_err"], rel=1e-12, abs=1e-300)
+        # a corrupted original: every changed finite value is outside the bound
+        x2 = x.copy()
+        idx = np.flatnonzero(np.isfinite(x2))[::501][:7]
+        x2[idx] = x2[idx] * 3 + 10
+        _, m2 = pk.decompress_verify(buf, torch.from_numpy(x2).cuda())
+        ref2 = _metrics_ref(x2, y_ref, bound, eps, P.range)
+        assert m2["violations"] == ref2["violations"]
+        if ci == 0:
+            assert m2["violations"] == len(idx)
