@@ -363,6 +363,29 @@ def run_ours(args):
                 "frac": algo / (dec_ms * 1e-3) / 1e9 / peak,
                 "traffic": traffic.get("decode") if world == 1 else None}
 
+    # ---- full-size bound check on the GPU: verify-mode decode of this rank's stream
+    # against the input (pfpl_decompress_verify), timed separately ----
+    verify = None
+    if world == 1:
+        ctypes_m = pk.Metrics()
+        tv = []
+        for _ in range(3):
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ob = ctypes.c_uint64(nbytes)
+            ev0.record(stream)
+            pk._check(L.pfpl_decompress_verify(out.data_ptr(), state["bytes"], x.data_ptr(), y.data_ptr(),
+                                               ctypes.byref(ob), ctypes.byref(ctypes_m), sh))
+            ev1.record(stream)
+            torch.cuda.synchronize()
+            tv.append(ev0.elapsed_time(ev1))
+        verify = {"violations": int(ctypes_m.violations), "max_abs_err": ctypes_m.max_abs_err,
+                  "max_rel_err": ctypes_m.max_rel_err, "psnr_db": ctypes_m.psnr,
+                  "n_finite": int(ctypes_m.n_finite), "eps": args.eps, "bound": args.bound,
+                  "decompress_verify_gbs": nbytes / (statistics.median(tv) * 1e-3) / 1e9,
+                  "what": "every value of the full-size stream decoded and checked against the input "
+                          "in the decode epilogue (f64 arithmetic); includes the API's host syncs"}
+        verify["encoder_stats"] = pk.last_stats(stream)     # the last timed compress on this stream
+
     # ---- end to end through the public API with host buffers (pinned) ----
     xh = x.cpu().pin_memory()
     oh = torch.empty(cap, dtype=torch.uint8).pin_memory()
@@ -416,6 +439,8 @@ def run_ours(args):
         "gpu_launches": int(launches), "launches_per_step": launches / args.steps,
         "clocks": clk.summary(), "wall_s": t_wall, "e2e": e2e, "context": PAPER_CONTEXT,
     }
+    if verify is not None:
+        line["verify"] = verify
     if world > 1:
         line["config"]["global_shape"] = list(spec.shape)
     if not args.no_cpu_baseline and world == 1:
