@@ -25,6 +25,12 @@
 
 namespace pfpl {
 
+#ifndef PFPL_DEC_LUT
+#define PFPL_DEC_LUT 1     // PRMT-selector gathers (+8% NYX, +17% rough decode)
+#endif
+#ifndef PFPL_DEC_WORCHK
+#define PFPL_DEC_WORCHK 0
+#endif
 #ifndef PFPL_DEC_IO_NS
 #define PFPL_DEC_IO_NS 1024       // the IO warp runs up to 8 chunks ahead: poll rarely
 #endif
@@ -50,6 +56,8 @@ struct DecShared {
     DecEntry q[NQD];
     unsigned long long full[NQD], empty[NQD];
     uint32_t tail;                     // ring bytes released by the compute warps (monotone)
+    uint32_t sel[16];                  // PRMT selector spreading popc(n) packed bytes to mask n
+    uint32_t selr[16];                 // same, unset bits repeating the previous byte (carry = 4)
 };
 constexpr int DOUT = 0;                // swizzled output staging (1024-aligned)
 constexpr int DRING = 16384;
@@ -104,7 +112,8 @@ __device__ __forceinline__ void dec1_count(const uint8_t* m1, DecShared& S, int 
 template <typename T, int KL, int KH>
 __device__ __forceinline__ void dec1_gather(uint32_t (&lo)[32], uint32_t (&hi)[32], const uint8_t* z1,
                                            int lane, const uint32_t (&nb)[64],
-                                           const uint32_t (&ex)[16], uint32_t offl, uint32_t offh) {
+                                           const uint32_t (&ex)[16], uint32_t offl, uint32_t offh,
+                                           const uint32_t* sel) {
     constexpr int NP = KL + KH;
 #pragma unroll
     for (int j = 0; j < NP; ++j) {
@@ -117,10 +126,23 @@ __device__ __forceinline__ void dec1_gather(uint32_t (&lo)[32], uint32_t (&hi)[3
             if (j < KL) lo[j] = 0; else hi[j - KL] = 0;
             continue;
         }
+#if PFPL_DEC_LUT
+        // the lane's popc(n) bytes are contiguous at z1 + o: one unaligned 4-byte read
+        // (two aligned words; the ring keeps >= 16 bytes of slack after a payload) and
+        // one PRMT that spreads them to the byte positions set in n (selector from sel[])
+        {
+            const uint8_t* pz = z1 + o;
+            const uint32_t mis = smem_u32(pz) & 3u;
+            const uint32_t* wp = (const uint32_t*)(pz - mis);
+            w = __byte_perm(__funnelshift_r(wp[0], wp[1], 8u * mis), 0u, sel[n]);
+        }
+        (void)r;
+#else
         if (n & 1u) w |= (uint32_t)z1[r++];
         if (n & 2u) w |= (uint32_t)z1[r++] << 8;
         if (n & 4u) w |= (uint32_t)z1[r++] << 16;
         if (n & 8u) w |= (uint32_t)z1[r] << 24;
+#endif
         if (j < KL) lo[j] = w; else hi[j - KL] = w;
     }
     if constexpr (KL > 0) transpose_inv<KL>(lo);
@@ -236,6 +258,22 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         }
         S.tail = 0;
         fence_barrier_init();
+    }
+    if (tid < 16) {
+        // selector nibble j: rank of byte j among the set bits of n, or 4 (a zero byte)
+        uint32_t v = 0, k = 0;
+        for (int j = 0; j < 4; ++j) v |= (((uint32_t)tid >> j) & 1u ? k++ : 4u) << (4 * j);
+        S.sel[tid] = v;
+        // repeat form: byte j = the last new byte at or before j, else the carry (byte 4)
+        uint32_t vr = 0, last = 4u;
+        k = 0;
+        for (int j = 0; j < 4; ++j) {
+            if (((uint32_t)tid >> j) & 1u) last = k++;
+            vr |= last << (4 * j);
+        }
+        S.selr[tid] = vr;
+    }
+    if (tid == 0) {
         prefetch_tmap(&tmap);
     }
     __syncthreads();
@@ -422,6 +460,25 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
 #pragma unroll
                 for (int i = 0; i < NB2 / 4; ++i) wv[i] = b * 0x01010101u;
             } else {
+#if PFPL_DEC_LUT
+                // 4 M1 bytes at a time: the new (non-repeated) bytes of the group are
+                // contiguous in Z2; one unaligned read and one PRMT whose selector (selr[])
+                // takes byte j from the group's k-th new byte, or repeats the byte before
+                // the group (the carry, operand byte 4) -- repeat elimination's inverse
+                uint32_t carry = base ? (uint32_t)z2[base - 1] : 0u;
+                uint32_t r0 = base;
+#pragma unroll
+                for (int i = 0; i < NB2 / 4; ++i) {
+                    const uint32_t nib = (bits >> (4 * i)) & 0xFu;
+                    const uint8_t* pz = z2 + r0;
+                    const uint32_t mis = smem_u32(pz) & 3u;
+                    const uint32_t* wp = (const uint32_t*)(pz - mis);
+                    const uint32_t w = __byte_perm(__funnelshift_r(wp[0], wp[1], 8u * mis), carry, S.selr[nib]);
+                    wv[i] = w;
+                    carry = w >> 24;
+                    r0 += __popc(nib);
+                }
+#else
 #pragma unroll
                 for (int i = 0; i < NB2 / 4; ++i) {
                     uint32_t w = 0;
@@ -433,6 +490,7 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                     }
                     wv[i] = w;
                 }
+#endif
             }
 #pragma unroll
             for (int i = 0; i < NB2 / 4; i += 4)
@@ -486,7 +544,7 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         const uint8_t* z1 = z2 + n2;
         const bool consistent = 4 + n4 + n3 + n2 + n1 == md.size;
         uint32_t lo[32], hi[32];
-        PFPL_DEC_TIER(dec1_gather, lo, hi, z1, lane, nb, ex, offl, offh);
+        PFPL_DEC_TIER(dec1_gather, lo, hi, z1, lane, nb, ex, offl, offh, S.sel);
 
         // ---- residual decode + delta decoder's inclusive scan ----
         W dq[32];
@@ -531,9 +589,11 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             if constexpr (sizeof(T) == 4 && MODE == MODE_ABS) {
                 if (fastdq) {
                     // all words of this thread are bins (the common case): no raw-word select
-                    W wor = 0;
+                    W wor = PFPL_DEC_WORCHK ? 0u : 0x00800000u;
+#if PFPL_DEC_WORCHK
 #pragma unroll
                     for (int i = 0; i < 32; ++i) wor |= (W)(carry + dq[i]);
+#endif
                     if (wor < 0x00800000u)
                         emit([&](W w) { return (T)q.abs_dq_bins((uint32_t)w, c23); });
                     else
