@@ -422,12 +422,32 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         const uint32_t n3 = __shfl_sync(PFPL_FULL, inc3, 31);
         const uint8_t* z3 = z4 + n4;
         uint32_t m2lo = 0, m2hi = 0;                            // M2 bytes 8*lane .. 8*lane+7
+#if PFPL_DEC_LUT
+        {
+            // two 4-byte groups, each one unaligned read + one repeat-selector PRMT
+            const uint32_t e3 = inc3 - cnt3;
+            uint32_t carry = e3 ? (uint32_t)z3[e3 - 1] : 0u;
+            uint32_t r0 = e3;
+#pragma unroll
+            for (int g = 0; g < 2; ++g) {
+                const uint32_t nib = (m3 >> (4 * g)) & 0xFu;
+                const uint8_t* pz = z3 + r0;
+                const uint32_t mis = smem_u32(pz) & 3u;
+                const uint32_t* wp = (const uint32_t*)(pz - mis);
+                const uint32_t w = __byte_perm(__funnelshift_r(wp[0], wp[1], 8u * mis), carry, S.selr[nib]);
+                if (g == 0) m2lo = w; else m2hi = w;
+                carry = w >> 24;
+                r0 += __popc(nib);
+            }
+        }
+#else
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
             const uint32_t cj = inc3 - cnt3 + __popc(m3 & ((2u << j) - 1u));
             const uint32_t bv = cj ? z3[cj - 1] : 0u;
             if (j < 4) m2lo |= bv << (8 * j); else m2hi |= bv << (8 * (j - 4));
         }
+#endif
         const uint32_t pc2 = __popc(m2lo) + __popc(m2hi);
         const uint32_t inc2 = warp_incl_scan(pc2, lane);
         const uint32_t n2 = __shfl_sync(PFPL_FULL, inc2, 31);
