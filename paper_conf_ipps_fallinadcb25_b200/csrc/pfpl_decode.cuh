@@ -58,6 +58,7 @@ struct DecShared {
     uint32_t tail;                     // ring bytes released by the compute warps (monotone)
     uint32_t sel[16];                  // PRMT selector spreading popc(n) packed bytes to mask n
     uint32_t selr[16];                 // same, unset bits repeating the previous byte (carry = 4)
+    unsigned long long vacc[8];        // verify mode: the CTA's metric accumulators (layout of p.vm)
 };
 constexpr int DOUT = 0;                // swizzled output staging (1024-aligned)
 constexpr int DRING = 16384;
@@ -195,7 +196,10 @@ struct VerAcc {
             const double d = fabs(xd - yd);
             mabs = fmax(mabs, d);
             ssq += d * d;
-            if (xd != 0.0) mrel = fmax(mrel, d / fabs(xd));
+            // divide only for candidates: q > mrel implies d > mrel*|x|*(1 - 2^-40), so the
+            // filter never drops a new maximum (the quotient itself is exact IEEE)
+            const double ax = fabs(xd);
+            if (ax != 0.0 && d > mrel * ax * 0.9999999999990905) mrel = fmax(mrel, d / ax);
             vmin = fmin(vmin, xd);
             vmax = fmax(vmax, xd);
             nfin += 1;
@@ -203,6 +207,48 @@ struct VerAcc {
             if (!(d <= lim)) nviol += 1;
         } else if (!((isnan(xd) && isnan(yd)) || xd == yd)) {
             nviol += 1;
+        }
+    }
+    // per chunk: warp-reduce into the CTA's shared accumulators and restart, so nothing
+    // stays live across the chunk loop (the kernel is register-bound)
+    __device__ __forceinline__ void flush_chunk(unsigned long long* sv) {
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) {
+            mabs = fmax(mabs, __shfl_xor_sync(PFPL_FULL, mabs, d));
+            mrel = fmax(mrel, __shfl_xor_sync(PFPL_FULL, mrel, d));
+            ssq += __shfl_xor_sync(PFPL_FULL, ssq, d);
+            vmin = fmin(vmin, __shfl_xor_sync(PFPL_FULL, vmin, d));
+            vmax = fmax(vmax, __shfl_xor_sync(PFPL_FULL, vmax, d));
+            nviol += __shfl_xor_sync(PFPL_FULL, nviol, d);
+            nfin += __shfl_xor_sync(PFPL_FULL, nfin, d);
+        }
+        if ((threadIdx.x & 31) == 0 && nfin + nviol) {
+            atomicMax(&sv[0], (unsigned long long)d2u(mabs));
+            atomicMax(&sv[1], (unsigned long long)d2u(mrel));
+            atomicAdd((double*)&sv[2], ssq);
+            atomicAdd(&sv[3], nviol);
+            atomicAdd(&sv[4], nfin);
+            if (nfin) {
+                atomicMin(&sv[5], ord_u64(vmin));
+                atomicMax(&sv[6], ord_u64(vmax));
+            }
+        }
+        mabs = mrel = ssq = 0.0;
+        vmin = INFINITY;
+        vmax = -INFINITY;
+        nviol = nfin = 0;
+    }
+    // once per CTA: shared accumulators -> global
+    static __device__ __forceinline__ void flush_cta(const unsigned long long* sv, const DecParams& p) {
+        if (sv[4] + sv[3] == 0) return;
+        atomicMax(&p.vm[0], sv[0]);
+        atomicMax(&p.vm[1], sv[1]);
+        atomicAdd((double*)&p.vm[2], u2d(sv[2]));
+        if (sv[3]) atomicAdd(&p.vm[3], sv[3]);
+        atomicAdd(&p.vm[4], sv[4]);
+        if (sv[4]) {
+            atomicMin(&p.vm[5], sv[5]);
+            atomicMax(&p.vm[6], sv[6]);
         }
     }
     __device__ __forceinline__ void flush(const DecParams& p) {
@@ -232,7 +278,8 @@ struct VerAcc {
 template <typename T>
 struct VerNone {
     __device__ __forceinline__ void add(T, T, const DecParams&) {}
-    __device__ __forceinline__ void flush(const DecParams&) {}
+    __device__ __forceinline__ void flush_chunk(unsigned long long*) {}
+    static __device__ __forceinline__ void flush_cta(const unsigned long long*, const DecParams&) {}
 };
 
 template <typename T, int MODE, bool MSR, bool VER = false>
@@ -272,6 +319,8 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             vr |= last << (4 * j);
         }
         S.selr[tid] = vr;
+        if (tid < 8)   // zeros; min = order(+inf), max = order(-inf)
+            S.vacc[tid] = tid == 5 ? 0xFFF0000000000000ull : tid == 6 ? ~0xFFF0000000000000ull : 0ull;
     }
     if (tid == 0) {
         prefetch_tmap(&tmap);
@@ -407,6 +456,7 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             if constexpr (VER) {       // the chunk's words were written by the whole CTA
                 for (uint32_t e = tid; e < m; e += NTC)
                     vacc.add(orig[c * (uint64_t)CW + e], ((const T*)dstc)[e], p);
+                vacc.flush_chunk(S.vacc);
             }
             continue;
         }
@@ -649,19 +699,22 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 bulk_commit();
             }
             if constexpr (VER) {
-                // this thread's staged rows against the originals (16-byte loads; each
-                // sector of the original chunk is read once)
+                // the staged chunk against the originals: thread t takes the 16-byte pieces
+                // t, t + NTC, ... of the chunk, so every load instruction of a warp reads
+                // 512 contiguous bytes (the staged piece q sits in row q/8, swizzled)
 #pragma unroll 1
                 for (int i = 0; i < 2 * S_; ++i) {
-                    const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
-                    const uint4 v = *(const uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4));
-                    const uint4 o = ldg_nc_v4(orig + c * (uint64_t)CW + (uint64_t)(r * (128 / S_) + (i & 7) * (16 / S_)));
+                    const int q = i * NTC + tid;                 // 16-byte piece of the chunk
+                    const int r = q >> 3;
+                    const uint4 v = *(const uint4*)(stage_out + r * 128 + (((q & 7) ^ (r & 7)) << 4));
+                    const uint4 o = ldg_nc_v4(orig + c * (uint64_t)CW + (uint64_t)q * (16 / S_));
                     T y[16 / S_], x[16 / S_];
                     memcpy(y, &v, 16);
                     memcpy(x, &o, 16);
 #pragma unroll
                     for (int k = 0; k < 16 / S_; ++k) vacc.add(x[k], y[k], p);
                 }
+                vacc.flush_chunk(S.vacc);
             }
         } else {
             // tail chunk: plain stores of the first m values
@@ -674,9 +727,13 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                     if constexpr (VER) vacc.add(orig[c * (uint64_t)CW + e], yv, p);
                 }
             }
+            if constexpr (VER) vacc.flush_chunk(S.vacc);
         }
     }
-    if constexpr (VER) vacc.flush(p);
+    if constexpr (VER) {
+        named_sync(1, NTC);        // every compute warp has flushed its last chunk
+        if (tid == 0) decltype(vacc)::flush_cta(S.vacc, p);
+    }
     if (tid == 0) bulk_wait0();    // all TMA stores of this CTA complete before exit
 }
 
