@@ -52,9 +52,6 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #ifndef PFPL_STATS
 #define PFPL_STATS 1
 #endif
-#ifndef PFPL_QSMEM
-#define PFPL_QSMEM 0
-#endif
 #ifndef PFPL_TIER4
 #define PFPL_TIER4 0        // P <= 4 uses the 8-plane tier: less hot code (+7% NYX)
 #endif
@@ -473,7 +470,6 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             // biased words (quantize_b): q + bias; the bias cancels in q[i] - q[i-1]
             W qprev = (W)qbias;
             bool done = false;
-            bool clobbered = false;      // stage overwritten by the fast path: fall back to HBM
             if constexpr (sizeof(T) == 4 && (MODE == MODE_ABS || MODE == MODE_NOA)) {
                 if (m == CW && !raw) {
                     // fast path: no per-element select or raw word; the
@@ -482,47 +478,6 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     // 8 independent predicate chains (a single chain would serialise
                     // 64 dependent FSETPs per thread)
                     bool ok[8] = {true, true, true, true, true, true, true, true};
-#if PFPL_QSMEM
-                    // quantize the stage in place in a short rolled loop (1/4 of the
-                    // code: the hot loop then fits the instruction cache), then read
-                    // the biased words back for the residuals
-                    {
-                        float pv = 0.0f;
-                        if (tid > 0) {
-                            if (lane == 0) {
-                                pv = ((const float*)p.in)[c * (uint64_t)CW + 32 * tid - 1];
-                            } else {
-                                const int r = tid - 1;
-                                pv = *(const float*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 12);
-                            }
-                        }
-                        __syncwarp();
-                        uint8_t* const wb = smem + s * DATAB;
-#pragma unroll 2
-                        for (int i = 0; i < 8; ++i) {
-                            uint4* const a = (uint4*)(wb + tid * 128 + (((i & 7) ^ (tid & 7)) << 4));
-                            const uint4 v = *a;
-                            bool* o = ok + 4 * (i & 1);
-                            const uint32_t z0 = q.abs_qf(u2f(v.x), o[0]), z1 = q.abs_qf(u2f(v.y), o[1]);
-                            const uint32_t z2 = q.abs_qf(u2f(v.z), o[2]), z3 = q.abs_qf(u2f(v.w), o[3]);
-                            *a = make_uint4(z0, z1, z2, z3);
-                        }
-                        if (tid > 0) zp = q.abs_qf(pv, ok[7]);
-                        fence_proxy_async();       // the stage is refilled by TMA later
-                        clobbered = true;
-                    }
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        const uint4 v = *(const uint4*)(buf + tid * 128 + (((i & 7) ^ (tid & 7)) << 4));
-                        const uint32_t z0 = v.x, z1 = v.y, z2 = v.z, z3 = v.w;
-                        const uint32_t r0 = rcode<MSR>(z0 - zp), r1 = rcode<MSR>(z1 - z0);
-                        const uint32_t r2 = rcode<MSR>(z2 - z1), r3 = rcode<MSR>(z3 - z2);
-                        zp = z3;
-                        orw |= r0 | r1;
-                        orw |= r2 | r3;
-                        lo[4 * i] = r0; lo[4 * i + 1] = r1; lo[4 * i + 2] = r2; lo[4 * i + 3] = r3;
-                    }
-#else
                     if (tid > 0) {
                         const int r = tid - 1;
                         zp = q.abs_qf(*(const float*)(buf + r * 128 + ((7 ^ (r & 7)) << 4) + 12), ok[7]);
@@ -540,7 +495,6 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         orw |= r2 | r3;
                         lo[4 * i] = r0; lo[4 * i + 1] = r1; lo[4 * i + 2] = r2; lo[4 * i + 3] = r3;
                     }
-#endif
                     done = __all_sync(PFPL_FULL, ok[0] && ok[1] && ok[2] && ok[3] && ok[4] && ok[5] &&
                                                      ok[6] && ok[7]);
                     orv = (W)orw;
@@ -608,7 +562,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 }
             }
             if (done) {
-            } else if (!TWO_PASS && m == CW && !clobbered) {
+            } else if (!TWO_PASS && m == CW) {
                 if (tid > 0) {
                     T pv;
                     if (sizeof(T) == 4) {
@@ -640,8 +594,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 }
                 add_raw(nraw);
             } else {
-                // tail chunk (or a clobbered stage): plain loads; R12 pads with the last
-                // value -> zero residuals
+                // tail chunk: plain loads; R12 pads with the last value -> zero residuals
                 const T* src = (const T*)p.in + c * (uint64_t)CW;
                 if (tid > 0) qprev = quantize_b<T, MODE>(q, src[min(32 * tid - 1, (int)m - 1)], raw);
                 uint32_t nraw = 0;
