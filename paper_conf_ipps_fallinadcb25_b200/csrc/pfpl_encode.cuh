@@ -62,7 +62,6 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #define PFPL_LB_NS 1500
 #endif
 constexpr int NQ = PFPL_ENC_NQ;      // IO queue depth
-constexpr int ARENA = PFPL_ENC_ARENA; // circular payload arena (bytes, multiple of 16)
 
 // hand-off from the compute warps to the IO warp, one per chunk
 struct QEntry {
@@ -81,10 +80,23 @@ struct EncShared {
     unsigned long long full[NIN], mq_full[NQ], mq_empty[NQ];
 };
 constexpr int ARENA_OFF = NIN * DATAB;
-constexpr int SHARED_OFF = ARENA_OFF + ARENA + 64;
-constexpr int ENC_SMEM = SHARED_OFF + (int)sizeof(EncShared);
-static_assert(ENC_SMEM <= 233472 / PFPL_ENC_MINB - 1024, "PFPL_ENC_MINB CTAs per SM must fit in shared memory");
-static_assert(DATAB + 16 + ((PRE3 + 15) & ~15) <= ARENA, "the arena must hold a worst-case slice");
+// per element type: arena bytes, shared-memory layout and CTAs per SM (f64 CTAs have 2
+// compute warps, so more of them fit; f64 streams are smoother per byte)
+#ifndef PFPL_ENC_ARENA64
+#define PFPL_ENC_ARENA64 24576
+#endif
+#ifndef PFPL_ENC_MINB64
+#define PFPL_ENC_MINB64 5
+#endif
+template <typename T> struct EncCfg {
+    static constexpr int ARENA = sizeof(T) == 4 ? PFPL_ENC_ARENA : PFPL_ENC_ARENA64;
+    static constexpr int SHARED_OFF = ARENA_OFF + ARENA + 64;
+    static constexpr int SMEM = SHARED_OFF + (int)sizeof(EncShared);
+    static constexpr int MINB = sizeof(T) == 4 ? PFPL_ENC_MINB : PFPL_ENC_MINB64;
+    static_assert(SMEM <= 233472 / MINB - 1024, "MINB CTAs per SM must fit in shared memory");
+    static_assert(DATAB + 16 + ((PRE3 + 15) & ~15) <= ARENA, "the arena must hold a worst-case slice");
+};
+constexpr int ENC_SMEM = EncCfg<float>::SMEM;   // f32 layout (host code: enc_smem(dtype))
 
 __device__ __forceinline__ void put_u64(uint8_t* p, uint64_t v) {
 #pragma unroll
@@ -175,6 +187,7 @@ __device__ __forceinline__ uint32_t zroom(uint32_t n1) { return min(2048u, (uint
 __device__ __forceinline__ uint32_t slice_bytes(uint32_t n1, uint32_t n2) {
     return a16(n1) + a16(PRE3 + min(n2, zroom(n1)));
 }
+template <int ARENA>
 __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
     const uint32_t R = a16(n1) + a16(PRE3 + zroom(n1));     // worst case
     const uint32_t head0 = S.head;
@@ -291,15 +304,16 @@ __device__ __forceinline__ bool is_bin_word(typename Tr<T>::W w, typename Tr<T>:
 }
 
 template <typename T, int MODE, bool MSR>
-__global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_ENC_MINB : 5)
+__global__ void __launch_bounds__(Tr<T>::NT + 32, EncCfg<T>::MINB)
 encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
     constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;
     constexpr int NB2 = 2048 / NTC;     // level-2 bytes per compute thread (16 or 32)
     constexpr int NWD2 = NB2 / 4;
 
+    constexpr int ARENA = EncCfg<T>::ARENA;
     extern __shared__ __align__(1024) uint8_t smem[];
-    EncShared& S = *reinterpret_cast<EncShared*>(smem + SHARED_OFF);
+    EncShared& S = *reinterpret_cast<EncShared*>(smem + EncCfg<T>::SHARED_OFF);
     uint8_t* const arena = smem + ARENA_OFF;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint64_t C = p.C;
@@ -654,7 +668,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             offl = tot_h + sl - tl + myl;
             offh = sh - th + myh;
             n1 = tot_l + tot_h;
-            head = slice_start(S, n1, lane);
+            head = slice_start<ARENA>(S, n1, lane);
         }
         uint8_t* const z1 = arena + head % ARENA;
         PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);

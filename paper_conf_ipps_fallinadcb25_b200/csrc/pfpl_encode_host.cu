@@ -22,8 +22,10 @@ static void* pick_enc(int dtype, int mode, bool ms) {
 
 static int enc_threads(int dtype) { return (dtype == 0 ? Tr<float>::NT : Tr<double>::NT) + 32; }
 
-static cudaError_t prepare_enc(void* fn) {
-    return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, ENC_SMEM);
+static int enc_smem(int dtype) { return dtype == 0 ? EncCfg<float>::SMEM : EncCfg<double>::SMEM; }
+
+static cudaError_t prepare_enc(void* fn, int dtype) {
+    return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, enc_smem(dtype));
 }
 
 int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
@@ -34,8 +36,8 @@ int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         void* fn = pick_enc(dtype, mode, ms);
-        prepare_enc(fn);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, enc_threads(dtype), ENC_SMEM);
+        prepare_enc(fn, dtype);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, enc_threads(dtype), enc_smem(dtype));
         g = sms * (per > 0 ? per : 1);
     }
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
@@ -85,12 +87,12 @@ cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int 
     void* fn = pick_enc(dtype, mode, ms);
     static bool prepared[2][4][2] = {};
     if (!prepared[dtype][mode][ms]) {
-        e = prepare_enc(fn);
+        e = prepare_enc(fn, dtype);
         if (e != cudaSuccess) return e;
         prepared[dtype][mode][ms] = true;
     }
     void* args[] = {(void*)&p, (void*)&map};
-    return cudaLaunchKernel(fn, dim3(grid), dim3(enc_threads(dtype)), args, ENC_SMEM, s);
+    return cudaLaunchKernel(fn, dim3(grid), dim3(enc_threads(dtype)), args, enc_smem(dtype), s);
 }
 
 }  // namespace pfpl
