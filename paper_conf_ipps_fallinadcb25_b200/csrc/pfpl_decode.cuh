@@ -31,6 +31,9 @@ namespace pfpl {
 #ifndef PFPL_DEC_WORCHK
 #define PFPL_DEC_WORCHK 0
 #endif
+#ifndef PFPL_DEC_IO_HINT
+#define PFPL_DEC_IO_HINT 0
+#endif
 #ifndef PFPL_DEC_IO_NS
 #define PFPL_DEC_IO_NS 1024       // the IO warp runs up to 8 chunks ahead: poll rarely
 #endif
@@ -381,7 +384,11 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             head += R;
             // the IO warp runs up to NQD chunks ahead: waiting here is the common
             // case, so sleep between polls instead of spinning on the issue port
+#if PFPL_DEC_IO_HINT
+            mbar_wait_wd(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
+#else
             mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21, PFPL_DEC_IO_NS);
+#endif
             // bulk copy of the aligned superset, never past the last 16-byte
             // boundary of the stream; the remainder by the lanes
             const uint8_t* a0 = g - delta;
