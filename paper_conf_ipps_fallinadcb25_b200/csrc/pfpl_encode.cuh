@@ -52,6 +52,9 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #ifndef PFPL_STATS
 #define PFPL_STATS 1
 #endif
+#ifndef PFPL_MIN_TIER
+#define PFPL_MIN_TIER 8
+#endif
 #ifndef PFPL_TIER4
 #define PFPL_TIER4 0        // P <= 4 uses the 8-plane tier: less hot code (+7% NYX)
 #endif
@@ -278,7 +281,7 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
         if (P == 0) FN<T, 0, 0>(__VA_ARGS__);                                           \
         else if (B == 32 || P <= 32) {                                                  \
             if (PFPL_TIER4 && P <= 4) FN<T, 4, 0>(__VA_ARGS__);                         \
-            else if (P <= 8) FN<T, 8, 0>(__VA_ARGS__);                                  \
+            else if (P <= 8 && PFPL_MIN_TIER <= 8) FN<T, 8, 0>(__VA_ARGS__);            \
             else if (P <= 16) FN<T, 16, 0>(__VA_ARGS__);                                \
             else FN<T, 32, 0>(__VA_ARGS__);                                             \
         } else {                                                                        \
