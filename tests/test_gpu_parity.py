@@ -298,3 +298,37 @@ def test_decompress_verify_metrics(pk, orc, dt, bound):
         assert m2["violations"] == ref2["violations"]
         if ci == 0:
             assert m2["violations"] == len(idx)
+
+
+def test_full_size_16gib_sampled(pk, orc):
+    """BASELINE.json configs[4] (16 GiB f32, n = 2^32, ABS 1E-3) at full size on one GPU, in
+    bench's launch configuration: the size table must account for the whole stream, and
+    sampled chunks (first, last, 62 random) must be byte-identical to the oracle's encoding of
+    the same 4096 values (ABS constants depend only on eps, so a lone chunk's payload is the
+    chunk's payload in any stream) and decode to the oracle's values bit for bit."""
+    free, _ = torch.cuda.mem_get_info()
+    if free < 60 * 2**30:
+        pytest.skip("needs ~60 GiB of free device memory")
+    spec = synth.CONFIGS["big16g"]
+    x = synth.generate(spec, device="cuda")
+    n = x.numel()
+    assert n == 2**32
+    s = pk.compress(x, "abs", 1e-3)
+    C = n // 4096
+    table = s[48:48 + 4 * C].cpu().numpy().view(np.uint32).astype(np.int64)
+    offs = np.concatenate([[0], np.cumsum(table)])
+    base = 48 + 4 * C
+    assert base + int(offs[-1]) == s.numel()
+    y = pk.decompress(s)
+    rng = np.random.default_rng(4)
+    for c in [0, C - 1] + list(rng.integers(1, C - 1, size=62)):
+        c = int(c)
+        xc = x[c * 4096:(c + 1) * 4096].cpu().numpy()
+        ref = orc.compress(xc, "abs", 1e-3)
+        assert int(table[c]) == len(ref) - 52, c
+        got = s[base + int(offs[c]):base + int(offs[c + 1])].cpu().numpy().tobytes()
+        assert got == ref[52:], c
+        yc = y[c * 4096:(c + 1) * 4096].cpu().numpy()
+        assert np.array_equal(yc.view(np.uint32), orc.decompress(ref).view(np.uint32)), c
+    del x, y, s
+    torch.cuda.empty_cache()
