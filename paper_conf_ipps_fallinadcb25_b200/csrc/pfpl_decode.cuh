@@ -25,6 +25,10 @@
 
 namespace pfpl {
 
+#ifndef PFPL_TP_UNROLL_D
+#define PFPL_TP_UNROLL_D 1
+#endif
+constexpr int kTpUnrollD = PFPL_TP_UNROLL_D;
 #ifndef PFPL_DEC_LUT
 #define PFPL_DEC_LUT 1     // PRMT-selector gathers (+8% NYX, +17% rough decode)
 #endif
@@ -683,7 +687,7 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 // them in place in a rolled loop (unrolled over 32 values the code
                 // overflows the instruction cache; see the encoder's TWO_PASS)
                 emit([&](W w) { T y; memcpy(&y, &w, sizeof(T)); return y; });
-#pragma unroll 1
+#pragma unroll kTpUnrollD
                 for (int i = 0; i < 2 * S_; ++i) {
                     const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
                     uint4* const a = (uint4*)(stage_out + r * 128 + (((i & 7) ^ (r & 7)) << 4));

@@ -52,6 +52,10 @@ constexpr int PRE3 = 4 + 32 + 256;   // M4 + Z4 + Z3 at most
 #ifndef PFPL_STATS
 #define PFPL_STATS 1
 #endif
+#ifndef PFPL_TP_UNROLL
+#define PFPL_TP_UNROLL 1     // quantize loop of the REL/f64 paths (4 or 2 values per iteration)
+#endif
+constexpr int kTpUnroll = PFPL_TP_UNROLL;
 #ifndef PFPL_MIN_TIER
 #define PFPL_MIN_TIER 8
 #endif
@@ -541,7 +545,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     }
                     __syncwarp();
                     uint32_t nraw = 0;
-#pragma unroll 1
+#pragma unroll kTpUnroll
                     for (int i = 0; i < 2 * S_; ++i) {
                         const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
                         uint4* const a = (uint4*)(wbuf + r * 128 + (((i & 7) ^ (r & 7)) << 4));
