@@ -194,6 +194,21 @@ __device__ __forceinline__ uint32_t zroom(uint32_t n1) { return min(2048u, (uint
 __device__ __forceinline__ uint32_t slice_bytes(uint32_t n1, uint32_t n2) {
     return a16(n1) + a16(PRE3 + min(n2, zroom(n1)));
 }
+#ifndef PFPL_ARENA_WAIT_NOINLINE
+#define PFPL_ARENA_WAIT_NOINLINE 0
+#endif
+// out-of-line arena wait: until tail == head0 (arena empty) or tail >= need
+static __device__ __noinline__ void arena_wait(const uint32_t* tail, uint32_t head0, uint32_t need,
+                                               uint32_t head) {
+    const uint64_t t0 = globaltimer();
+    for (;;) {
+        const uint32_t t = ld_volatile_u32(tail);
+        if (t == head0 || (int32_t)(t - need) >= 0) return;
+        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x13, head);
+        __nanosleep(64);
+    }
+}
+
 template <int ARENA>
 __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
     const uint32_t R = a16(n1) + a16(PRE3 + zroom(n1));     // worst case
@@ -208,6 +223,9 @@ __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1,
         const uint32_t t = ld_volatile_u32(&S.tail);
         return t != head0 && head + R - t > (uint32_t)ARENA;
     };
+#if PFPL_ARENA_WAIT_NOINLINE
+    if (lane == 0 && full()) arena_wait(&S.tail, head0, head + R - (uint32_t)ARENA, head);
+#else
     if (lane == 0 && full()) {
         const uint64_t t0 = globaltimer();
         while (full()) {
@@ -215,6 +233,7 @@ __device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1,
             __nanosleep(64);
         }
     }
+#endif
     __syncwarp();
     return head;                                            // monotone byte counter
 }
