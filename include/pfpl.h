@@ -131,6 +131,30 @@ int pfpl_decompress_chunks(const void* hdr_host, const uint32_t* table_host,
                            uint64_t first_chunk, uint64_t n_chunks, const void* payload_dev,
                            uint64_t payload_bytes, void* out_dev, uint64_t cap, void* stream);
 
+/* ---- host-resident (out-of-core) arrays ----
+ * The array and the stream live in HOST memory (pinned for full PCIe rate;
+ * pageable works, slower) and may exceed HBM.  They are streamed through two
+ * device segment buffers of seg_chunks chunks each (0 = default 2048 chunks =
+ * 32 MiB): segment k+1's H2D and segment k-1's D2H (two library-owned copy
+ * streams) overlap segment k's kernel on `stream`.  Chunks are independent
+ * and payload offsets are a prefix sum of the chunk sizes,
+ * carried across segments on the host, so the stream is byte-identical to
+ * pfpl_compress of the same array on the device.  NOA makes one extra
+ * streaming pass for the global {min, max}.  The copy streams, events
+ * and about 4 * seg_chunks * 16 KiB of segment buffers are library-owned,
+ * cached per (device, stream) and grow-only.
+ * pfpl_compress_host: *out_bytes = capacity of out_host on entry (use
+ * pfpl_max_compressed_bytes), stream size on return; PFPL_ERR_CAPACITY if the
+ * stream would overflow (nothing is written past the capacity).
+ * pfpl_decompress_host: *out_bytes = capacity of out_host on entry, n*s on
+ * return; PFPL_ERR_CORRUPT for a table whose sizes exceed in_bytes.
+ * Both synchronise and return only after every copy has landed. */
+int pfpl_compress_host(const void* in_host, uint64_t n, int dtype, int bound, double eps,
+                       unsigned opts, void* out_host, uint64_t* out_bytes, uint64_t seg_chunks,
+                       void* stream);
+int pfpl_decompress_host(const void* in_host, uint64_t in_bytes, void* out_host,
+                         uint64_t* out_bytes, uint64_t seg_chunks, void* stream);
+
 /* ---- misc ---- */
 const char* pfpl_strerror(int status);
 int pfpl_last_cuda_error(void);

@@ -61,6 +61,8 @@ def lib():
             "pfpl_compress_shard": (i32, [vp, u64, u64, u64, i32, i32, dbl, ctypes.c_uint, vp, vp,
                                           u64, pu64, vp, vp]),
             "pfpl_decompress_chunks": (i32, [vp, vp, u64, u64, vp, u64, vp, u64, vp]),
+            "pfpl_compress_host": (i32, [vp, u64, i32, i32, dbl, ctypes.c_uint, vp, pu64, u64, vp]),
+            "pfpl_decompress_host": (i32, [vp, u64, vp, pu64, u64, vp]),
             "pfpl_strerror": (ctypes.c_char_p, [i32]),
             "pfpl_last_cuda_error": (i32, []),
             "pfpl_watchdog_report": (i32, [ctypes.POINTER(ctypes.c_uint)]),
@@ -264,6 +266,49 @@ def decompress_chunks(hdr: bytes, table, first_chunk: int, payload: torch.Tensor
                                       payload.numel(), out.data_ptr(),
                                       out.numel() * out.element_size(), _stream(stream))
     _check(st, "decompress_chunks")
+
+
+def _require_host(t: torch.Tensor, name: str):
+    if t.is_cuda or not t.is_contiguous():
+        raise PFPLError(-1, f"{name} must be a contiguous host tensor")
+
+
+def compress_host(x: torch.Tensor, bound="abs", eps: float = 1e-3, ms: bool = False,
+                  out: torch.Tensor | None = None, seg_chunks: int = 0, stream=None) -> torch.Tensor:
+    """Compress a float32/float64 HOST tensor (pinned for full PCIe rate) through the
+    pipelined out-of-core path (pfpl_compress_host); returns a uint8 host tensor (a
+    view of `out` if given; a pinned one is allocated otherwise)."""
+    _require_host(x, "x")
+    dt = _dtype_code(x)
+    n = x.numel()
+    if out is None:
+        out = torch.empty(max_compressed_bytes(n, dt), dtype=torch.uint8, pin_memory=True)
+    _require_host(out, "out")
+    nbytes = ctypes.c_uint64(out.numel())
+    st = lib().pfpl_compress_host(x.data_ptr() if n else None, n, dt, _bound(bound), float(eps),
+                                  OPT_MS if ms else 0, out.data_ptr(), ctypes.byref(nbytes),
+                                  seg_chunks, _stream(stream))
+    _check(st, "compress_host")
+    return out[:nbytes.value]
+
+
+def decompress_host(buf: torch.Tensor, out: torch.Tensor | None = None, seg_chunks: int = 0,
+                    stream=None) -> torch.Tensor:
+    """Decompress a uint8 HOST tensor holding a stream into a host tensor
+    (pfpl_decompress_host)."""
+    _require_host(buf, "buf")
+    if buf.numel() < HEADER_BYTES:
+        raise PFPLError(-4, "stream shorter than its header")
+    h = peek_header(buf[:HEADER_BYTES].numpy().tobytes())
+    tdt = torch.float32 if h["dtype"] == F32 else torch.float64
+    if out is None:
+        out = torch.empty(max(h["n"], 1), dtype=tdt, pin_memory=True)
+    _require_host(out, "out")
+    ob = ctypes.c_uint64(out.numel() * out.element_size())
+    st = lib().pfpl_decompress_host(buf.data_ptr(), buf.numel(), out.data_ptr(), ctypes.byref(ob),
+                                    seg_chunks, _stream(stream))
+    _check(st, "decompress_host")
+    return out[:h["n"]]
 
 
 def last_stats(stream=None) -> dict:

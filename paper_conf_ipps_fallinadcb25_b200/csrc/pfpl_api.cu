@@ -386,6 +386,10 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
 
 }  // namespace
 
+namespace pfpl {
+int record_cuda_error(int e) { return cuda_fail((cudaError_t)e); }
+}  // namespace pfpl
+
 extern "C" {
 
 uint64_t pfpl_max_compressed_bytes(uint64_t n, int dtype) {

@@ -103,4 +103,7 @@ int decode_tickets_per_cta();
 float log2p_host_f32(float a);
 double log2p_host_f64(double a);
 
+// records e as the last CUDA error (pfpl_last_cuda_error) and returns PFPL_ERR_CUDA
+int record_cuda_error(int e);
+
 }  // namespace pfpl
