@@ -155,6 +155,21 @@ int pfpl_compress_host(const void* in_host, uint64_t n, int dtype, int bound, do
 int pfpl_decompress_host(const void* in_host, uint64_t in_bytes, void* out_host,
                          uint64_t* out_bytes, uint64_t seg_chunks, void* stream);
 
+/* ---- multi-field batches (e.g. CESM's 33 fields) ----
+ * Compresses `count` independent device arrays (same dtype, bound and eps)
+ * into `count` independent streams, each byte-identical to pfpl_compress of
+ * that array.  The fields are forked over 4 library-owned non-blocking
+ * streams (cached per (device, stream)) so consecutive small fields overlap
+ * each other's launch ramp-up and drain, and joined back onto `stream`.
+ * in[f], out[f]: device pointers, 16-B aligned; out_bytes[f] (host array):
+ * capacity of out[f] on entry, stream size on return.  Synchronises once.
+ * Returns the first error (argument errors before anything is enqueued;
+ * PFPL_ERR_CAPACITY if any field overflowed -- its out_bytes entry is then
+ * left at its capacity). */
+int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int dtype, int bound,
+                        double eps, unsigned opts, void* const* out, uint64_t* out_bytes,
+                        void* stream);
+
 /* ---- misc ---- */
 const char* pfpl_strerror(int status);
 int pfpl_last_cuda_error(void);

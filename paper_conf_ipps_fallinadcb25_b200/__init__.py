@@ -63,6 +63,7 @@ def lib():
             "pfpl_decompress_chunks": (i32, [vp, vp, u64, u64, vp, u64, vp, u64, vp]),
             "pfpl_compress_host": (i32, [vp, u64, i32, i32, dbl, ctypes.c_uint, vp, pu64, u64, vp]),
             "pfpl_decompress_host": (i32, [vp, u64, vp, pu64, u64, vp]),
+            "pfpl_compress_batch": (i32, [i32, vp, vp, i32, i32, dbl, ctypes.c_uint, vp, vp, vp]),
             "pfpl_strerror": (ctypes.c_char_p, [i32]),
             "pfpl_last_cuda_error": (i32, []),
             "pfpl_watchdog_report": (i32, [ctypes.POINTER(ctypes.c_uint)]),
@@ -266,6 +267,32 @@ def decompress_chunks(hdr: bytes, table, first_chunk: int, payload: torch.Tensor
                                       payload.numel(), out.data_ptr(),
                                       out.numel() * out.element_size(), _stream(stream))
     _check(st, "decompress_chunks")
+
+
+def compress_batch(xs: list, bound="abs", eps: float = 1e-3, ms: bool = False,
+                   outs: list | None = None, stream=None) -> list:
+    """Compress a list of same-dtype CUDA tensors in one call (pfpl_compress_batch);
+    returns one uint8 CUDA tensor (stream) per field."""
+    if not xs:
+        return []
+    for x in xs:
+        _require_cuda(x, "xs[i]")
+    dt = _dtype_code(xs[0])
+    if any(_dtype_code(x) != dt for x in xs):
+        raise PFPLError(-1, "compress_batch: all fields must share one dtype")
+    k = len(xs)
+    if outs is None:
+        outs = [torch.empty(max_compressed_bytes(x.numel(), dt), dtype=torch.uint8, device=x.device)
+                for x in xs]
+    ins = (ctypes.c_void_p * k)(*[x.data_ptr() for x in xs])
+    ns = (ctypes.c_uint64 * k)(*[x.numel() for x in xs])
+    os_ = (ctypes.c_void_p * k)(*[o.data_ptr() for o in outs])
+    caps = (ctypes.c_uint64 * k)(*[o.numel() for o in outs])
+    with torch.cuda.device(xs[0].device):
+        st = lib().pfpl_compress_batch(k, ins, ns, dt, _bound(bound), float(eps),
+                                       OPT_MS if ms else 0, os_, caps, _stream(stream))
+    _check(st, "compress_batch")
+    return [o[:caps[i]] for i, o in enumerate(outs)]
 
 
 def _require_host(t: torch.Tensor, name: str):

@@ -1,0 +1,118 @@
+// pfpl_batch.cu -- many independent fields in one call (SURVEY 8(f) NEXT-4:
+// multi-field batches such as CESM's 33 per-timestep fields).  A small
+// field (CESM: 1,583 chunks, 26 MB) keeps the persistent encoder busy for only
+// ~2 chunks per CTA, so one field per launch is bound by ramp-up and drain.
+// The batch forks the fields over a cached pool of non-blocking streams so
+// consecutive fields' launches overlap each other's tails, then joins back
+// onto the caller's stream with one D2H of every stream size.  Each field's
+// stream is exactly pfpl_compress's (same kernel, same arguments).
+#include <cuda_runtime.h>
+
+#include <map>
+#include <mutex>
+#include <utility>
+
+#include "../../include/pfpl.h"
+#include "pfpl_internal.h"
+
+using namespace pfpl;
+
+namespace {
+
+constexpr int kLanes = 4;
+
+struct Lanes {
+    cudaStream_t st[kLanes] = {};
+    cudaEvent_t done[kLanes] = {};
+    cudaEvent_t fork = nullptr;
+    uint64_t* res_dev = nullptr;    // 2 words per field (pfpl_compress_async's result)
+    uint64_t* res_host = nullptr;
+    int res_cap = 0;
+};
+
+std::mutex g_mu;
+std::map<std::pair<int, void*>, Lanes*> g_lanes;
+
+#define BK(x)                                                       \
+    do {                                                            \
+        cudaError_t _e = (x);                                       \
+        if (_e != cudaSuccess) return record_cuda_error((int)_e);   \
+    } while (0)
+
+int get_lanes(cudaStream_t s, int count, Lanes** out) {
+    int dev = 0;
+    BK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    Lanes*& L = g_lanes[{dev, (void*)s}];
+    if (!L) {
+        L = new Lanes();
+        for (int i = 0; i < kLanes; ++i) {
+            BK(cudaStreamCreateWithFlags(&L->st[i], cudaStreamNonBlocking));
+            BK(cudaEventCreateWithFlags(&L->done[i], cudaEventDisableTiming));
+        }
+        BK(cudaEventCreateWithFlags(&L->fork, cudaEventDisableTiming));
+    }
+    if (count > L->res_cap) {
+        BK(cudaStreamSynchronize(s));
+        if (L->res_dev) BK(cudaFree(L->res_dev));
+        if (L->res_host) BK(cudaFreeHost(L->res_host));
+        L->res_dev = nullptr;
+        L->res_host = nullptr;
+        L->res_cap = 0;
+        BK(cudaMalloc((void**)&L->res_dev, 16ull * count));
+        BK(cudaMallocHost((void**)&L->res_host, 16ull * count));
+        L->res_cap = count;
+    }
+    *out = L;
+    return PFPL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int dtype, int bound,
+                        double eps, unsigned opts, void* const* out, uint64_t* out_bytes,
+                        void* stream) {
+    if (count < 0 || (count && (!in || !n || !out || !out_bytes))) return PFPL_ERR_ARG;
+    if (count == 0) return PFPL_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    Lanes* L = nullptr;
+    int st = get_lanes(s, count, &L);
+    if (st != PFPL_OK) return st;
+    BK(cudaEventRecord(L->fork, s));
+    const int lanes = count < kLanes ? count : kLanes;
+    for (int i = 0; i < lanes; ++i) BK(cudaStreamWaitEvent(L->st[i], L->fork, 0));
+    int first_err = PFPL_OK;
+    for (int f = 0; f < count; ++f) {
+        st = pfpl_compress_async(in[f], n[f], dtype, bound, eps, opts, out[f], out_bytes[f],
+                                 L->res_dev + 2 * f, L->st[f % lanes]);
+        if (st != PFPL_OK) {
+            first_err = st;
+            break;
+        }
+    }
+    // join every lane (also after an error, so nothing is left in flight)
+    for (int i = 0; i < lanes; ++i) {
+        BK(cudaEventRecord(L->done[i], L->st[i]));
+        BK(cudaStreamWaitEvent(s, L->done[i], 0));
+    }
+    if (first_err != PFPL_OK) {
+        BK(cudaStreamSynchronize(s));
+        return first_err;
+    }
+    BK(cudaMemcpyAsync(L->res_host, L->res_dev, 16ull * count, cudaMemcpyDeviceToHost, s));
+    BK(cudaStreamSynchronize(s));
+    for (int f = 0; f < count; ++f) {
+        const uint64_t total = L->res_host[2 * f];
+        const int code = (int)(int32_t)(uint32_t)L->res_host[2 * f + 1];
+        if (code != 0 || total > out_bytes[f]) {
+            if (first_err == PFPL_OK) first_err = code ? code : PFPL_ERR_CAPACITY;
+        } else {
+            out_bytes[f] = total;
+        }
+    }
+    return first_err;
+}
+
+}  // extern "C"

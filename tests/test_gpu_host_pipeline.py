@@ -74,3 +74,31 @@ def test_host_pipeline_errors(pk):
     with pytest.raises(pk.PFPLError) as ei:
         pk.decompress_host(bad)
     assert ei.value.code == -4
+
+
+@pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_compress_batch_matches_oracle(pk, orc, bound, dt):
+    """pfpl_compress_batch: every field's stream equals the oracle's for that
+    field alone (fields of mixed sizes, an empty one, ragged tails; more fields
+    than internal streams so lanes are reused)."""
+    cw = 4096 if dt == np.float32 else 2048
+    sizes = [3 * cw + 5, 0, 1, cw, 11 * cw + 777, 2 * cw - 1, 5]
+    xs = []
+    for i, n in enumerate(sizes):
+        spec = synth.FieldSpec("t", (max(n, 1),), "f32" if dt == np.float32 else "f64", 20 + i,
+                               A=0.5, tau=0.01)
+        xs.append(synth.generate(spec).numpy()[:n].copy())
+    outs = pk.compress_batch([torch.from_numpy(x).cuda() for x in xs], bound, 1e-3)
+    for x, o in zip(xs, outs):
+        assert o.cpu().numpy().tobytes() == orc.compress(x, bound, 1e-3), (bound, dt, x.size)
+
+
+def test_compress_batch_capacity(pk):
+    xs = [torch.randn(30000, device="cuda") for _ in range(3)]
+    outs = [torch.empty(pk.max_compressed_bytes(30000, torch.float32), dtype=torch.uint8, device="cuda")
+            for _ in range(3)]
+    outs[1] = outs[1][:1000]
+    with pytest.raises(pk.PFPLError) as ei:
+        pk.compress_batch(xs, "abs", 1e-3, outs=outs)
+    assert ei.value.code == -3
