@@ -8,6 +8,7 @@
 // stream is exactly pfpl_compress's (same kernel, same arguments).
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <map>
 #include <mutex>
 #include <utility>
@@ -19,11 +20,21 @@ using namespace pfpl;
 
 namespace {
 
-constexpr int kLanes = 4;
+constexpr int kMaxLanes = 16;
+
+// lanes (internal streams) a batch forks over; PFPL_BATCH_LANES overrides (tuning)
+int lanes_cfg() {
+    static int v = [] {
+        const char* e = getenv("PFPL_BATCH_LANES");
+        int x = e ? atoi(e) : 4;
+        return x < 1 ? 1 : (x > kMaxLanes ? kMaxLanes : x);
+    }();
+    return v;
+}
 
 struct Lanes {
-    cudaStream_t st[kLanes] = {};
-    cudaEvent_t done[kLanes] = {};
+    cudaStream_t st[kMaxLanes] = {};
+    cudaEvent_t done[kMaxLanes] = {};
     cudaEvent_t fork = nullptr;
     uint64_t* res_dev = nullptr;    // 2 words per field (pfpl_compress_async's result)
     uint64_t* res_host = nullptr;
@@ -46,7 +57,7 @@ int get_lanes(cudaStream_t s, int count, Lanes** out) {
     Lanes*& L = g_lanes[{dev, (void*)s}];
     if (!L) {
         L = new Lanes();
-        for (int i = 0; i < kLanes; ++i) {
+        for (int i = 0; i < kMaxLanes; ++i) {
             BK(cudaStreamCreateWithFlags(&L->st[i], cudaStreamNonBlocking));
             BK(cudaEventCreateWithFlags(&L->done[i], cudaEventDisableTiming));
         }
@@ -81,7 +92,7 @@ int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int
     int st = get_lanes(s, count, &L);
     if (st != PFPL_OK) return st;
     BK(cudaEventRecord(L->fork, s));
-    const int lanes = count < kLanes ? count : kLanes;
+    const int lanes = count < lanes_cfg() ? count : lanes_cfg();
     for (int i = 0; i < lanes; ++i) BK(cudaStreamWaitEvent(L->st[i], L->fork, 0));
     int first_err = PFPL_OK;
     for (int f = 0; f < count; ++f) {
