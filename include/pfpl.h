@@ -169,6 +169,14 @@ int pfpl_decompress_host(const void* in_host, uint64_t in_bytes, void* out_host,
 int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int dtype, int bound,
                         double eps, unsigned opts, void* const* out, uint64_t* out_bytes,
                         void* stream);
+/* Decompresses `count` independent streams (device pointers in[f], in_bytes[f]
+ * bytes each) into out[f] (device, 16-B aligned; out_bytes[f] = capacity on
+ * entry, n*s on return).  The headers come back in one round trip, the fields
+ * are forked over the same 4 streams; each output equals pfpl_decompress's.
+ * Synchronises twice.  Returns the first error (PFPL_ERR_CORRUPT for a stream
+ * shorter than its header or a corrupt table/payload). */
+int pfpl_decompress_batch(int count, const void* const* in, const uint64_t* in_bytes,
+                          void* const* out, uint64_t* out_bytes, void* stream);
 
 /* ---- misc ---- */
 const char* pfpl_strerror(int status);

@@ -64,6 +64,7 @@ def lib():
             "pfpl_compress_host": (i32, [vp, u64, i32, i32, dbl, ctypes.c_uint, vp, pu64, u64, vp]),
             "pfpl_decompress_host": (i32, [vp, u64, vp, pu64, u64, vp]),
             "pfpl_compress_batch": (i32, [i32, vp, vp, i32, i32, dbl, ctypes.c_uint, vp, vp, vp]),
+            "pfpl_decompress_batch": (i32, [i32, vp, vp, vp, vp, vp]),
             "pfpl_strerror": (ctypes.c_char_p, [i32]),
             "pfpl_last_cuda_error": (i32, []),
             "pfpl_watchdog_report": (i32, [ctypes.POINTER(ctypes.c_uint)]),
@@ -293,6 +294,32 @@ def compress_batch(xs: list, bound="abs", eps: float = 1e-3, ms: bool = False,
                                        OPT_MS if ms else 0, os_, caps, _stream(stream))
     _check(st, "compress_batch")
     return [o[:caps[i]] for i, o in enumerate(outs)]
+
+
+def decompress_batch(bufs: list, outs: list | None = None, stream=None) -> list:
+    """Decompress a list of uint8 CUDA tensors (streams) in one call
+    (pfpl_decompress_batch); returns one tensor per stream."""
+    if not bufs:
+        return []
+    for b in bufs:
+        _require_cuda(b, "bufs[i]")
+        if b.numel() < HEADER_BYTES:
+            raise PFPLError(-4, "stream shorter than its header")
+    k = len(bufs)
+    if outs is None:
+        outs = []
+        for b in bufs:
+            h = peek_header(b[:HEADER_BYTES].cpu().numpy().tobytes())
+            tdt = torch.float32 if h["dtype"] == F32 else torch.float64
+            outs.append(torch.empty(max(h["n"], 1), dtype=tdt, device=b.device))
+    ins = (ctypes.c_void_p * k)(*[b.data_ptr() for b in bufs])
+    nb = (ctypes.c_uint64 * k)(*[b.numel() for b in bufs])
+    os_ = (ctypes.c_void_p * k)(*[o.data_ptr() for o in outs])
+    caps = (ctypes.c_uint64 * k)(*[o.numel() * o.element_size() for o in outs])
+    with torch.cuda.device(bufs[0].device):
+        st = lib().pfpl_decompress_batch(k, ins, nb, os_, caps, _stream(stream))
+    _check(st, "decompress_batch")
+    return [o[:caps[i] // o.element_size()] for i, o in enumerate(outs)]
 
 
 def _require_host(t: torch.Tensor, name: str):

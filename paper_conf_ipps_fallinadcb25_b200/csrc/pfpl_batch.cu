@@ -1,4 +1,4 @@
-// pfpl_batch.cu -- many independent fields in one call (SURVEY 8(f) NEXT-4:
+// pfpl_batch.cu -- many independent fields in one call (compress and decompress) (SURVEY 8(f) NEXT-4:
 // multi-field batches such as CESM's 33 per-timestep fields).  A small
 // field (CESM: 1,583 chunks, 26 MB) keeps the persistent encoder busy for only
 // ~2 chunks per CTA, so one field per launch is bound by ramp-up and drain.
@@ -39,6 +39,8 @@ struct Lanes {
     uint64_t* res_dev = nullptr;    // 2 words per field (pfpl_compress_async's result)
     uint64_t* res_host = nullptr;
     int res_cap = 0;
+    uint8_t* hdr_host = nullptr;    // kHeaderBytes per field (decompress)
+    int hdr_cap = 0;
 };
 
 std::mutex g_mu;
@@ -75,6 +77,17 @@ int get_lanes(cudaStream_t s, int count, Lanes** out) {
         L->res_cap = count;
     }
     *out = L;
+    return PFPL_OK;
+}
+
+int ensure_hdr(Lanes* L, cudaStream_t s, int count) {
+    if (count <= L->hdr_cap) return PFPL_OK;
+    BK(cudaStreamSynchronize(s));
+    if (L->hdr_host) BK(cudaFreeHost(L->hdr_host));
+    L->hdr_host = nullptr;
+    L->hdr_cap = 0;
+    BK(cudaMallocHost((void**)&L->hdr_host, (size_t)kHeaderBytes * count));
+    L->hdr_cap = count;
     return PFPL_OK;
 }
 
@@ -122,6 +135,61 @@ int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int
         } else {
             out_bytes[f] = total;
         }
+    }
+    return first_err;
+}
+
+int pfpl_decompress_batch(int count, const void* const* in, const uint64_t* in_bytes,
+                          void* const* out, uint64_t* out_bytes, void* stream) {
+    if (count < 0 || (count && (!in || !in_bytes || !out || !out_bytes))) return PFPL_ERR_ARG;
+    if (count == 0) return PFPL_OK;
+    for (int f = 0; f < count; ++f)
+        if (!in[f] || in_bytes[f] < kHeaderBytes) return PFPL_ERR_CORRUPT;
+    cudaStream_t s = (cudaStream_t)stream;
+    Lanes* L = nullptr;
+    int st = get_lanes(s, count, &L);
+    if (st == PFPL_OK) st = ensure_hdr(L, s, count);
+    if (st != PFPL_OK) return st;
+    // every header in one round trip (n and dtype size each output)
+    for (int f = 0; f < count; ++f)
+        BK(cudaMemcpyAsync(L->hdr_host + (size_t)kHeaderBytes * f, in[f], kHeaderBytes,
+                           cudaMemcpyDeviceToHost, s));
+    BK(cudaStreamSynchronize(s));
+    BK(cudaEventRecord(L->fork, s));
+    const int lanes = count < lanes_cfg() ? count : lanes_cfg();
+    for (int i = 0; i < lanes; ++i) BK(cudaStreamWaitEvent(L->st[i], L->fork, 0));
+    int first_err = PFPL_OK;
+    for (int f = 0; f < count; ++f) {
+        st = pfpl_decompress_async(in[f], in_bytes[f], L->hdr_host + (size_t)kHeaderBytes * f,
+                                   out[f], out_bytes[f], L->res_dev + 2 * f, L->st[f % lanes]);
+        if (st != PFPL_OK) {
+            first_err = st;
+            break;
+        }
+    }
+    for (int i = 0; i < lanes; ++i) {
+        BK(cudaEventRecord(L->done[i], L->st[i]));
+        BK(cudaStreamWaitEvent(s, L->done[i], 0));
+    }
+    if (first_err != PFPL_OK) {
+        BK(cudaStreamSynchronize(s));
+        return first_err;
+    }
+    BK(cudaMemcpyAsync(L->res_host, L->res_dev, 16ull * count, cudaMemcpyDeviceToHost, s));
+    BK(cudaStreamSynchronize(s));
+    for (int f = 0; f < count; ++f) {
+        const int code = (int)(int32_t)(uint32_t)L->res_host[2 * f + 1];
+        if (code != 0) {
+            if (first_err == PFPL_OK) first_err = code;
+            continue;
+        }
+        uint64_t n = 0;
+        int dtype = 0, bound = 0;
+        double eps = 0;
+        unsigned flags = 0;
+        pfpl_peek_header(L->hdr_host + (size_t)kHeaderBytes * f, kHeaderBytes, &n, &dtype, &bound,
+                         &eps, &flags);
+        out_bytes[f] = n * (dtype == PFPL_F32 ? 4u : 8u);
     }
     return first_err;
 }

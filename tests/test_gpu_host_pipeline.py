@@ -90,8 +90,13 @@ def test_compress_batch_matches_oracle(pk, orc, bound, dt):
                                A=0.5, tau=0.01)
         xs.append(synth.generate(spec).numpy()[:n].copy())
     outs = pk.compress_batch([torch.from_numpy(x).cuda() for x in xs], bound, 1e-3)
-    for x, o in zip(xs, outs):
-        assert o.cpu().numpy().tobytes() == orc.compress(x, bound, 1e-3), (bound, dt, x.size)
+    refs = [orc.compress(x, bound, 1e-3) for x in xs]
+    for x, o, r in zip(xs, outs, refs):
+        assert o.cpu().numpy().tobytes() == r, (bound, dt, x.size)
+    # pfpl_decompress_batch on the oracle's streams gives the oracle's values
+    ys = pk.decompress_batch([torch.frombuffer(bytearray(r), dtype=torch.uint8).cuda() for r in refs])
+    for x, y, r in zip(xs, ys, refs):
+        assert np.array_equal(_bits(y.cpu().numpy()), _bits(orc.decompress(r))), (bound, dt, x.size)
 
 
 def test_compress_batch_capacity(pk):
@@ -102,3 +107,14 @@ def test_compress_batch_capacity(pk):
     with pytest.raises(pk.PFPLError) as ei:
         pk.compress_batch(xs, "abs", 1e-3, outs=outs)
     assert ei.value.code == -3
+
+
+def test_decompress_batch_corrupt(pk):
+    xs = [torch.randn(30000, device="cuda") for _ in range(3)]
+    outs = [o.clone() for o in pk.compress_batch(xs, "abs", 1e-3)]
+    with pytest.raises(pk.PFPLError) as ei:
+        pk.decompress_batch([outs[0], outs[1][:-5], outs[2]])
+    assert ei.value.code == -4
+    ys = pk.decompress_batch(outs)
+    for x, y in zip(xs, ys):
+        assert torch.equal(y, pk.decompress(pk.compress(x, "abs", 1e-3)))

@@ -18,18 +18,31 @@ outs = [torch.empty(pk.max_compressed_bytes(x.numel(), torch.float32), dtype=tor
         for x in xs]
 res = {}
 for bound in ("abs", "noa", "rel"):
-    seq, bat = [], []
+    seq, bat, dseq, dbat = [], [], [], []
+    ys = [torch.empty_like(x) for x in xs]
     for it in range(6):
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         a = [pk.compress(x, bound, 1e-3, out=o).numel() for x, o in zip(xs, outs)]
         t1 = time.perf_counter()
-        b = [o.numel() for o in pk.compress_batch(xs, bound, 1e-3, outs=outs)]
+        bs = pk.compress_batch(xs, bound, 1e-3, outs=outs)
         t2 = time.perf_counter()
+        b = [o.numel() for o in bs]
         assert a == b
+        torch.cuda.synchronize()
+        t3 = time.perf_counter()
+        for s_, y in zip(bs, ys):
+            pk.decompress(s_, out=y)
+        t4 = time.perf_counter()
+        pk.decompress_batch(bs, outs=ys)
+        t5 = time.perf_counter()
         if it:
             seq.append(t1 - t0)
             bat.append(t2 - t1)
+            dseq.append(t4 - t3)
+            dbat.append(t5 - t4)
     res[bound] = {"sequential_gbs": nbytes / statistics.median(seq) / 1e9,
-                  "batch_gbs": nbytes / statistics.median(bat) / 1e9, "ratio": nbytes / sum(b)}
+                  "batch_gbs": nbytes / statistics.median(bat) / 1e9, "ratio": nbytes / sum(b),
+                  "decompress_sequential_gbs": nbytes / statistics.median(dseq) / 1e9,
+                  "decompress_batch_gbs": nbytes / statistics.median(dbat) / 1e9}
 print(json.dumps({"fields": 33, "bytes": nbytes, "eps": 1e-3, **res}))
