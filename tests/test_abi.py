@@ -77,3 +77,15 @@ def test_product_never_imports_oracle():
                         assert not (node.module or "").startswith("oracle"), f
             if f.endswith((".cu", ".cuh", ".h")):
                 assert "oracle" not in open(os.path.join(dirpath, f)).read().lower(), f
+
+
+def test_batch_and_host_bindings_need_no_gpu_for_empty_and_reject_cuda_only_args():
+    """Python-side argument handling of the NEXT-4 bindings (no compute call)."""
+    import torch
+    import paper_conf_ipps_fallinadcb25_b200 as pk
+    assert pk.compress_batch([]) == []
+    assert pk.decompress_batch([]) == []
+    with pytest.raises(pk.PFPLError):
+        pk.compress_host(torch.zeros(8, 2).t(), "abs", 1e-3)     # non-contiguous host tensor
+    with pytest.raises(pk.PFPLError):
+        pk.compress_batch([torch.zeros(8)], "abs", 1e-3)       # host tensor where CUDA is required
