@@ -185,7 +185,9 @@ int pfpl_last_cuda_error(void);
  * the call returns PFPL_ERR_CUDA), copies {site, block, thread, detail} to
  * out4 and returns 1; otherwise returns 0. */
 int pfpl_watchdog_report(unsigned int* out4);
-/* Frees the calling thread's scratch for the current device. */
+/* Frees the library's cached scratch for the current device: per-stream
+ * look-back/result scratch, the host-pipeline buffers and copy streams, and
+ * the batch lanes.  Synchronises the device; later calls re-create them. */
 int pfpl_release_scratch(void);
 /* Reconstruction-quality metrics of a decompression against the original values
  * (the paper's Fig. 16 analogue), accumulated in the

@@ -659,6 +659,8 @@ int pfpl_watchdog_report(unsigned int* out4) {
 int pfpl_release_scratch(void) {
     int dev = 0;
     CK(cudaGetDevice(&dev));
+    release_pipes(dev);
+    release_lanes(dev);
     std::lock_guard<std::mutex> lk(g_mu);
     for (auto it = g_scratch.begin(); it != g_scratch.end();) {
         if (it->first.first != dev) { ++it; continue; }

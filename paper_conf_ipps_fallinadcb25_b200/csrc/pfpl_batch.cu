@@ -93,6 +93,23 @@ int ensure_hdr(Lanes* L, cudaStream_t s, int count) {
 
 }  // namespace
 
+void pfpl::release_lanes(int dev) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    for (auto it = g_lanes.begin(); it != g_lanes.end();) {
+        if (it->first.first != dev) { ++it; continue; }
+        Lanes* L = it->second;
+        cudaDeviceSynchronize();
+        for (int i = 0; i < kMaxLanes; ++i) {
+            if (L->st[i]) cudaStreamDestroy(L->st[i]);
+            if (L->done[i]) cudaEventDestroy(L->done[i]);
+        }
+        if (L->fork) cudaEventDestroy(L->fork);
+        cudaFree(L->res_dev); cudaFreeHost(L->res_host); cudaFreeHost(L->hdr_host);
+        delete L;
+        it = g_lanes.erase(it);
+    }
+}
+
 extern "C" {
 
 int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int dtype, int bound,

@@ -105,5 +105,8 @@ double log2p_host_f64(double a);
 
 // records e as the last CUDA error (pfpl_last_cuda_error) and returns PFPL_ERR_CUDA
 int record_cuda_error(int e);
+// free the host-pipeline (pfpl_pipeline.cu) and batch-lane (pfpl_batch.cu) caches of device dev
+void release_pipes(int dev);
+void release_lanes(int dev);
 
 }  // namespace pfpl

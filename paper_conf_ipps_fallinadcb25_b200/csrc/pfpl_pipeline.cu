@@ -124,6 +124,24 @@ inline uint64_t tsz_of(int dtype) { return dtype == PFPL_F32 ? 4u : 8u; }
 
 }  // namespace
 
+void pfpl::release_pipes(int dev) {
+    std::lock_guard<std::mutex> lk(g_pipe_mu);
+    for (auto it = g_pipes.begin(); it != g_pipes.end();) {
+        if (it->first.first != dev) { ++it; continue; }
+        Pipe* p = it->second;
+        cudaDeviceSynchronize();
+        for (int b = 0; b < 2; ++b) {
+            cudaFree(p->inbuf[b]); cudaFree(p->outbuf[b]);
+            cudaEventDestroy(p->in_ready[b]); cudaEventDestroy(p->in_free[b]);
+            cudaEventDestroy(p->out_free[b]);
+        }
+        if (p->h2d) cudaStreamDestroy(p->h2d);
+        if (p->d2h) cudaStreamDestroy(p->d2h);
+        delete p;
+        it = g_pipes.erase(it);
+    }
+}
+
 extern "C" {
 
 int pfpl_compress_host(const void* in_host, uint64_t n, int dtype, int bound, double eps,

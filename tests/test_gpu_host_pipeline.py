@@ -118,3 +118,16 @@ def test_decompress_batch_corrupt(pk):
     ys = pk.decompress_batch(outs)
     for x, y in zip(xs, ys):
         assert torch.equal(y, pk.decompress(pk.compress(x, "abs", 1e-3)))
+
+
+def test_release_scratch_then_reuse(pk):
+    """pfpl_release_scratch frees the pipeline and lane caches; the next calls
+    re-create them and give the same bytes."""
+    x = torch.randn(70000, dtype=torch.float32)
+    a = pk.compress_host(x, "abs", 1e-3, seg_chunks=2).clone()
+    b = [o.cpu() for o in pk.compress_batch([x.cuda(), x[:5000].cuda()], "noa", 1e-3)]
+    assert pk.lib().pfpl_release_scratch() == 0
+    assert torch.equal(pk.compress_host(x, "abs", 1e-3, seg_chunks=2), a)
+    b2 = [o.cpu() for o in pk.compress_batch([x.cuda(), x[:5000].cuda()], "noa", 1e-3)]
+    assert all(torch.equal(u, v) for u, v in zip(b, b2))
+    assert torch.equal(pk.decompress_host(a), pk.decompress(a.cuda()).cpu())
