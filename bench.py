@@ -12,18 +12,23 @@ so no flush is needed.  Times are CUDA events on the launching stream,
 max over ranks.  value = compression throughput in uncompressed GB/s (10^9,
 P:225), whole job; decompression GB/s and ratio are reported beside it.
 
-N > 1 (torchrun, one process per GPU): weak scaling -- rank r compresses
-chunk-aligned slab r of an (N*512)x512x512 field; NCCL all-reduces the NOA
-range (NOA only) and all-gathers the per-shard payload sizes so every rank
-knows its offset in the single assembled stream.
+N > 1 (one process per GPU; `--gpus N` starts the N ranks itself under
+torch.distributed.run when WORLD_SIZE is unset): BASELINE.json configs[4] --
+the 16 GiB f32 field (1024x2048x2048, n = 2^32), ABS 1E-3, STRONG scaling:
+rank r generates and compresses its chunk-aligned slab; NCCL all-reduces the
+NOA range (NOA only) and all-gathers the per-shard payload sizes so every
+rank knows its offset in the single assembled stream.  After
+the timed region rank 0 compresses the whole field on one GPU and every
+rank's table slice and payload are compared (64-bit checksums of the same
+byte ranges) with that single-GPU stream.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
-import subprocess
 import sys
 import threading
 import time
@@ -42,7 +47,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="nyx")
+    ap.add_argument("--config", default=None,
+                    help="synth config; default nyx (configs[1]) at N=1, big16g (configs[4]) at N>1")
     ap.add_argument("--bound", default="abs")
     ap.add_argument("--eps", type=float, default=1e-3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -120,10 +126,40 @@ class Clocks:
                 "samples": len(self.samples), "source": "NVML, polled during the timed region"}
 
 
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def _time_oracle(x, bound, eps, threads, seconds):
+    """Median-free mean over enough repetitions to fill ~`seconds` (at least 1)."""
+    import oracle
+    t0 = time.perf_counter()
+    s = oracle.compress(x, bound, eps, nthreads=threads)
+    first = time.perf_counter() - t0
+    reps = max(1, min(50, int(seconds / max(first, 1e-3))))
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        oracle.compress(x, bound, eps, nthreads=threads)
+    tc = (time.perf_counter() - t0) / reps
+    rd = max(1, reps // 2)
+    t0 = time.perf_counter()
+    for _ in range(rd):
+        oracle.decompress(s, nthreads=threads)
+    td = (time.perf_counter() - t0) / rd
+    return tc, td, s, reps
+
+
 def cpu_baseline(spec, bound, eps, seconds):
-    """The oracle as it stands (plain C, chunks over all host threads) on a
-    bounded sample of the same workload: the first rows of the field."""
-    import numpy as np
+    """The oracle as it stands (plain C, chunks over host threads) on a bounded
+    sample of the same workload (the first rows of the field), on the SAME bytes
+    twice: one thread, and all host threads (OpenMP over chunks) -- SURVEY 8(d)."""
     import oracle
     import synth
     cores = len(os.sched_getaffinity(0))
@@ -131,23 +167,19 @@ def cpu_baseline(spec, bound, eps, seconds):
     inner = spec.n // spec.shape[0]
     rows = max(1, min(spec.shape[0], (64 << 20) // (inner * spec.itemsize)))
     x = synth.generate(spec, slab=(0, rows)).numpy()
-    t0 = time.perf_counter()
-    s = oracle.compress(x, bound, eps, nthreads=cores)
-    t1 = time.perf_counter()
-    reps = max(1, int(seconds / max(t1 - t0, 1e-3)))
-    reps = min(reps, 50)
-    t0 = time.perf_counter()
-    for _ in range(reps):
-        oracle.compress(x, bound, eps, nthreads=cores)
-    tc = (time.perf_counter() - t0) / reps
-    t0 = time.perf_counter()
-    for _ in range(max(1, reps // 2)):
-        oracle.decompress(s, nthreads=cores)
-    td = (time.perf_counter() - t0) / max(1, reps // 2)
+    tc, td, s, reps = _time_oracle(x, bound, eps, cores, 0.6 * seconds)
+    # single thread on a quarter of the same sample (whole rows), so the run stays bounded
+    x1 = x[:max(inner, (x.size // 4) // inner * inner)]
+    tc1, td1, _, reps1 = _time_oracle(x1, bound, eps, 1, 0.4 * seconds)
     return {"value": x.nbytes / tc / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "cpu_model": cpu_model(),
             "sample": f"first {rows} of {spec.shape[0]} rows ({x.nbytes / 1e6:.1f} MB), "
-                      f"{reps} reps, OpenMP over chunks",
-            "decompress_gbs": x.nbytes / td / 1e9, "ratio": x.nbytes / len(s)}
+                      f"{reps} reps, OpenMP over chunks on {cores} threads",
+            "decompress_gbs": x.nbytes / td / 1e9, "ratio": x.nbytes / len(s),
+            "single_thread": {"value": x1.nbytes / tc1 / 1e9, "unit": "GB/s", "cores": 1,
+                              "decompress_gbs": x1.nbytes / td1 / 1e9,
+                              "sample": f"first {x1.size // inner} rows ({x1.nbytes / 1e6:.1f} MB) "
+                                        f"of the same sample, {reps1} reps, 1 thread"}}
 
 
 def run_reference(args):
@@ -158,7 +190,7 @@ def run_reference(args):
     import numpy as np
     import oracle
     import synth
-    spec = synth.CONFIGS[args.config]
+    spec = synth.CONFIGS[args.config or ("nyx" if args.gpus == 1 else "big16g")]
     cores = len(os.sched_getaffinity(0))
     oracle.build()
     inner = spec.n // spec.shape[0]
@@ -181,9 +213,10 @@ def run_reference(args):
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": 1e3 * (statistics.median(tc) + statistics.median(td)),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": spec.dtype,
-        "data": "synthetic", "config": _config(spec, args, sample_rows=rows),
+        "data": "synthetic", "config": _config(spec, args, sample_rows=rows, world=args.gpus),
         "ratio": x.nbytes / len(s), "decompress_gbs": x.nbytes / statistics.median(td) / 1e9,
         "cpu_baseline": {"value": comp, "unit": "GB/s", "cores": cores, "kind": "oracle",
+                         "cpu_model": cpu_model(),
                          "sample": f"first {rows} of {spec.shape[0]} rows ({x.nbytes / 1e6:.1f} MB) per step"},
         "e2e": {"value": comp, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         "context": PAPER_CONTEXT,
@@ -203,11 +236,11 @@ def _traffic(config, bound):
     return dict(e, source=t.get("source")) if e else {}
 
 
-def _config(spec, args, sample_rows=None):
+def _config(spec, args, sample_rows=None, world=1):
     c = {"workload": f"{spec.name}, {args.bound.upper()} {args.eps:g}", "shape": list(spec.shape),
          "bound": args.bound, "eps": args.eps, "n": spec.n, "bytes": spec.nbytes,
          "l2": "inputs larger than L2 (no flush needed)" if spec.nbytes > 126e6 else "L2 flushed",
-         "parallelism": f"dp{args.gpus} chunk shards"}
+         "parallelism": f"dp{world} chunk shards"}
     if sample_rows is not None:
         c["sample_rows"] = sample_rows
     return c
@@ -246,16 +279,15 @@ def run_ours(args):
         dist.barrier()
     L = pk.lib()
 
-    # weak scaling: rank r owns slab r of an (N*rows) x ... field, chunk-aligned
-    base = synth.CONFIGS[args.config]
-    import dataclasses
-    spec = dataclasses.replace(base, shape=(base.shape[0] * world,) + tuple(base.shape[1:]))
+    # N = 1: the headline NYX field (configs[1]); N > 1: configs[4], the 16 GiB field,
+    # strong scaling -- rank r owns the chunk-aligned slab r of the same global field
+    cfg = args.config or ("nyx" if world == 1 else "big16g")
+    base = synth.CONFIGS[cfg]
+    spec = base
     n_total = spec.n
     esz = spec.itemsize
     fc, nch, e0, e1 = pdist.shard_chunks(n_total, esz, rank, world)
-    inner = n_total // spec.shape[0]
-    assert e0 % inner == 0 and e1 % inner == 0, "slabs must be whole rows"
-    x = synth.generate(spec, device=dev, slab=(e0 // inner, e1 // inner))
+    x = _generate_range(synth, spec, e0, e1, dev)
     torch.cuda.synchronize()
     n = x.numel()
     nbytes = n * esz
@@ -351,7 +383,7 @@ def run_ours(args):
     enc_ms = statistics.median(tc)
     my_comp = comp_bytes if world == 1 else (4 * nch + r.payload.numel())
     algo = nbytes + my_comp                  # input read + stream written, per launch (this rank)
-    traffic = _traffic(args.config, args.bound)
+    traffic = _traffic(cfg, args.bound)
     roof = {"bound": "hbm", "achieved": algo / (enc_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
             "frac": algo / (enc_ms * 1e-3) / 1e9 / peak,
             "traffic": traffic.get("encode") if world == 1 else None,
@@ -453,6 +485,12 @@ def run_ours(args):
                        "decompress_gbs the same for pfpl_decompress_host",
                "sequential_device_api": seq}
 
+    # ---- N > 1: the assembled stream must be the single-GPU stream ----
+    identity = None
+    if world > 1:
+        identity = _identity_check(pk, synth, pdist, dist, spec, args, state["shard"], out, nch,
+                                   rank, world, dev, stream)
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -461,8 +499,8 @@ def run_ours(args):
         "metric": METRIC, "value": comp_gbs, "unit": "GB/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": (tc_sum + td_sum) / args.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": spec.dtype, "data": "synthetic",
-        "config": _config(base, args),
+        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": spec.dtype,
+        "data": "synthetic", "config": _config(base, args, world=world),
         "ratio": ratio, "compress_gbs": comp_gbs, "decompress_gbs": dec_gbs,
         "compress_ms": tc_sum / args.steps, "decompress_ms": td_sum / args.steps,
         "roofline": roof, "roofline_decode": roof_dec,
@@ -473,6 +511,11 @@ def run_ours(args):
         line["verify"] = verify
     if world > 1:
         line["config"]["global_shape"] = list(spec.shape)
+        line["identity"] = identity
+        line["per_gpu_gbs"] = comp_gbs / world
+        if os.environ.get("PFPL_BENCH_SHARE_GPU"):
+            line["shared_gpu"] = ("functional run: all ranks share the visible GPU(s) "
+                                  f"({torch.cuda.device_count()}); not a scaling measurement")
     if not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_baseline(base, args.bound, args.eps, args.cpu_seconds)
     print(json.dumps(line), flush=True)
@@ -480,10 +523,102 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+def _generate_range(synth, spec, e0, e1, dev):
+    """Elements [e0, e1) of the field, generated from whole rows of its slowest axis."""
+    import torch
+    inner = spec.n // spec.shape[0]
+    r0, r1 = e0 // inner, -(-e1 // inner)
+    x = synth.generate(spec, device=dev, slab=(r0, r1))
+    if e0 - r0 * inner or r1 * inner - e1:
+        x = x[e0 - r0 * inner:e1 - r0 * inner].contiguous()
+    torch.cuda.synchronize()
+    return x
+
+
+def _cksum(t):
+    """(bytes, two 64-bit position-weighted sums) of a uint8 CUDA tensor."""
+    import torch
+    nb = t.numel()
+    pad = (-nb) % 8
+    v = torch.cat([t, torch.zeros(pad, dtype=torch.uint8, device=t.device)]) if pad else t
+    w = v.view(torch.int64)
+    idx = torch.arange(w.numel(), dtype=torch.int64, device=t.device)
+    h1 = int((w * (2 * idx + 1)).sum().item())
+    h2 = int((w ^ (idx * 40503 + 17)).sum().item())
+    return [nb, h1, h2]
+
+
+def _identity_check(pk, synth, pdist, dist, spec, args, r, out, nch, rank, world, dev, stream):
+    """Rank 0 compresses the whole field with the single-GPU API; every rank's
+    table slice and payload are compared with the same byte ranges of that
+    stream by 64-bit checksums (all-gathered), plus the header and total size."""
+    import torch
+    mine = _cksum(r.table.view(torch.uint8)) + _cksum(r.payload)
+    vals = torch.tensor(mine, dtype=torch.int64)
+    backend = dist.get_backend()
+    if backend == "nccl":
+        vals = vals.to(dev)
+    allv = [torch.empty_like(vals) for _ in range(world)]
+    dist.all_gather(allv, vals)
+    allv = [v.cpu().tolist() for v in allv]
+    res = None
+    if rank == 0:
+        t0 = time.perf_counter()
+        full = _generate_range(synth, spec, 0, spec.n, dev)
+        single = pk.compress(full, args.bound, args.eps, stream=stream)
+        torch.cuda.synchronize()
+        ok = len(r.header) == 48 and bytes(single[:48].cpu().numpy().tobytes()) == r.header
+        ok = ok and single.numel() == r.total_bytes
+        C = pdist.chunks_of(spec.n, spec.itemsize)
+        toff = 48
+        poff = 48 + 4 * C
+        per_rank = []
+        for q in range(world):
+            _, nq, _, _ = pdist.shard_chunks(spec.n, spec.itemsize, q, world)
+            tb = single[toff:toff + 4 * nq]
+            pb = single[poff:poff + r.sizes[q]]
+            good = (_cksum(tb) + _cksum(pb)) == allv[q]
+            per_rank.append(bool(good))
+            toff += 4 * nq
+            poff += r.sizes[q]
+        ok = ok and all(per_rank) and poff == single.numel()
+        res = {"identical_to_single_gpu_stream": bool(ok), "per_rank": per_rank,
+               "stream_bytes": int(single.numel()),
+               "method": "rank 0: pfpl_compress of the whole field on one GPU; header, total size and "
+                         "64-bit checksums of every rank's table slice and payload vs the same byte "
+                         "ranges of that stream",
+               "seconds": round(time.perf_counter() - t0, 2)}
+        del full, single
+        torch.cuda.empty_cache()
+    dist.barrier()
+    return res
+
+
+def relaunch_distributed(args) -> None:
+    """`--gpus N` without torchrun: start the N ranks ourselves (torch.distributed.run,
+    127.0.0.1).  With fewer visible GPUs than N, the ranks share them (gloo for the two
+    tiny exchanges) -- a functional run, flagged `shared_gpu` in the line."""
+    import torch
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ)
+    if torch.cuda.device_count() < args.gpus:
+        env["PFPL_BENCH_SHARE_GPU"] = "1"
+        env.setdefault("PFPL_DIST_BACKEND", "gloo")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr=127.0.0.1", f"--master-port={port}",
+           os.path.abspath(__file__)] + sys.argv[1:]
+    os.execve(sys.executable, cmd, env)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
+    elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch_distributed(args)
     else:
         run_ours(args)
 

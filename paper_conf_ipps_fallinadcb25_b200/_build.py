@@ -18,7 +18,7 @@ SRCS = sorted(f for f in glob.glob(os.path.join(PKG, "csrc", "*.cu")) if not f.e
 INST = os.path.join(PKG, "csrc", "pfpl_inst.cu")
 # (kind, dtype, mode): encoder f32/f64 x ABS/REL/RAW/NOA, decoder f32/f64 x ABS/REL/RAW
 INST_JOBS = [(0, d, m) for d in (0, 1) for m in range(4)] + [(1, d, m) for d in (0, 1) for m in range(3)]
-DEPS = SRCS + glob.glob(os.path.join(PKG, "csrc", "*.h")) + glob.glob(os.path.join(PKG, "csrc", "*.cuh")) \
+DEPS = SRCS + [INST] + glob.glob(os.path.join(PKG, "csrc", "*.h")) + glob.glob(os.path.join(PKG, "csrc", "*.cuh")) \
     + [os.path.join(ROOT, "include", "pfpl.h")]
 
 NVCC_FLAGS = [

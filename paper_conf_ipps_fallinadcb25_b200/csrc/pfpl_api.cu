@@ -8,6 +8,7 @@
 #include <atomic>
 #include <cfloat>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -49,12 +50,13 @@ std::map<std::pair<int, void*>, Scratch*> g_scratch;
 unsigned int* g_wd_host = nullptr;     // mapped pinned watchdog report {site, block, thread, detail}
 unsigned int* g_wd_dev = nullptr;
 
+std::once_flag g_wd_once;
 unsigned int* watchdog_ptr() {
-    if (!g_wd_host) {
-        if (cudaHostAlloc(&g_wd_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_wd_host = nullptr; return nullptr; }
+    std::call_once(g_wd_once, [] {
+        if (cudaHostAlloc(&g_wd_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_wd_host = nullptr; return; }
         memset(g_wd_host, 0, 64);
         if (cudaHostGetDevicePointer(&g_wd_dev, g_wd_host, 0) != cudaSuccess) g_wd_dev = nullptr;
-    }
+    });
     return g_wd_dev;
 }
 
@@ -88,17 +90,19 @@ int get_scratch(cudaStream_t s, uint64_t C, Scratch** out) {
         CK(cudaMalloc(&sc->stats, 4 * sizeof(unsigned long long)));
         CK(cudaMemsetAsync(sc->stats, 0, 4 * sizeof(unsigned long long), s));
     }
+    // look-back descriptors: one per chunk (encoder) / per 1024-chunk tile (size scan)
+    auto desc_words = [](uint64_t cap) { return cap; };
     if (C > sc->status_cap) {
         if (sc->status) CK(cudaFreeAsync(sc->status, s));
         uint64_t cap = C < 1024 ? 1024 : C + C / 4;
-        CK(cudaMallocAsync(&sc->status, cap * sizeof(unsigned long long), s));
-        CK(cudaMemsetAsync(sc->status, 0, cap * sizeof(unsigned long long), s));
+        CK(cudaMallocAsync(&sc->status, desc_words(cap) * sizeof(unsigned long long), s));
+        CK(cudaMemsetAsync(sc->status, 0, desc_words(cap) * sizeof(unsigned long long), s));
         sc->status_cap = cap;
         sc->epoch = 0;
     }
     // epochs tag look-back descriptors so no per-call memset is needed
     if (++sc->epoch >= 0xFFFFu) {
-        CK(cudaMemsetAsync(sc->status, 0, sc->status_cap * sizeof(unsigned long long), s));
+        CK(cudaMemsetAsync(sc->status, 0, desc_words(sc->status_cap) * sizeof(unsigned long long), s));
         sc->epoch = 1;
     }
     *out = sc;
@@ -388,6 +392,31 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
 
 namespace pfpl {
 int record_cuda_error(int e) { return cuda_fail((cudaError_t)e); }
+
+int grid_limit() {
+    static const int v = [] {
+        const char* e = getenv("PFPL_GRID_LIMIT");
+        const long x = e ? atol(e) : 0;
+        return x > 0 ? (int)(x < (1 << 30) ? x : (1 << 30)) : (1 << 30);
+    }();
+    return v;
+}
+
+// every argument check pfpl_compress_async makes before enqueueing anything
+int check_compress_args(const void* in, uint64_t n, int dtype, int bound, double eps,
+                        unsigned opts, const void* out, uint64_t cap) {
+    if (dtype != PFPL_F32 && dtype != PFPL_F64) return PFPL_ERR_ARG;
+    if (bound != PFPL_ABS && bound != PFPL_REL && bound != PFPL_NOA) return PFPL_ERR_ARG;
+    if (n > (1ull << 40)) return PFPL_ERR_ARG;
+    if ((n && !in) || !out) return PFPL_ERR_ARG;
+    if (!aligned16(in) || !aligned16(out)) return PFPL_ERR_ALIGN;
+    QConst qc;
+    int mode = 0;
+    const int st = host_qconst(dtype, bound, eps, opts, &qc, &mode);
+    if (st != PFPL_OK) return st;
+    if (cap < kHeaderBytes + 4 * chunks_of(n, dtype)) return PFPL_ERR_CAPACITY;
+    return PFPL_OK;
+}
 }  // namespace pfpl
 
 extern "C" {

@@ -33,6 +33,7 @@ int lanes_cfg() {
 }
 
 struct Lanes {
+    std::mutex mu;                  // held for a whole batch call (one user of res/hdr at a time)
     cudaStream_t st[kMaxLanes] = {};
     cudaEvent_t done[kMaxLanes] = {};
     cudaEvent_t fork = nullptr;
@@ -52,13 +53,8 @@ std::map<std::pair<int, void*>, Lanes*> g_lanes;
         if (_e != cudaSuccess) return record_cuda_error((int)_e);   \
     } while (0)
 
-int get_lanes(cudaStream_t s, int count, Lanes** out) {
-    int dev = 0;
-    BK(cudaGetDevice(&dev));
-    std::lock_guard<std::mutex> lk(g_mu);
-    Lanes*& L = g_lanes[{dev, (void*)s}];
-    if (!L) {
-        L = new Lanes();
+int init_lanes(Lanes* L, cudaStream_t s, int count, Lanes** out) {
+    if (!L->fork) {
         for (int i = 0; i < kMaxLanes; ++i) {
             BK(cudaStreamCreateWithFlags(&L->st[i], cudaStreamNonBlocking));
             BK(cudaEventCreateWithFlags(&L->done[i], cudaEventDisableTiming));
@@ -78,6 +74,18 @@ int get_lanes(cudaStream_t s, int count, Lanes** out) {
     }
     *out = L;
     return PFPL_OK;
+}
+
+int get_lanes(cudaStream_t s, int count, Lanes** out, std::unique_lock<std::mutex>* own) {
+    int dev = 0;
+    BK(cudaGetDevice(&dev));
+    std::unique_lock<std::mutex> lk(g_mu);
+    Lanes*& L = g_lanes[{dev, (void*)s}];
+    if (!L) L = new Lanes();
+    Lanes* const Lp = L;
+    lk.unlock();
+    *own = std::unique_lock<std::mutex>(Lp->mu);     // two threads on one stream are serialised
+    return init_lanes(Lp, s, count, out);
 }
 
 int ensure_hdr(Lanes* L, cudaStream_t s, int count) {
@@ -117,9 +125,15 @@ int pfpl_compress_batch(int count, const void* const* in, const uint64_t* n, int
                         void* stream) {
     if (count < 0 || (count && (!in || !n || !out || !out_bytes))) return PFPL_ERR_ARG;
     if (count == 0) return PFPL_OK;
+    // every field's argument errors before anything is enqueued (pfpl.h)
+    for (int f = 0; f < count; ++f) {
+        const int e = check_compress_args(in[f], n[f], dtype, bound, eps, opts, out[f], out_bytes[f]);
+        if (e != PFPL_OK) return e;
+    }
     cudaStream_t s = (cudaStream_t)stream;
     Lanes* L = nullptr;
-    int st = get_lanes(s, count, &L);
+    std::unique_lock<std::mutex> own;
+    int st = get_lanes(s, count, &L, &own);
     if (st != PFPL_OK) return st;
     BK(cudaEventRecord(L->fork, s));
     const int lanes = count < lanes_cfg() ? count : lanes_cfg();
@@ -164,7 +178,8 @@ int pfpl_decompress_batch(int count, const void* const* in, const uint64_t* in_b
         if (!in[f] || in_bytes[f] < kHeaderBytes) return PFPL_ERR_CORRUPT;
     cudaStream_t s = (cudaStream_t)stream;
     Lanes* L = nullptr;
-    int st = get_lanes(s, count, &L);
+    std::unique_lock<std::mutex> own;
+    int st = get_lanes(s, count, &L, &own);
     if (st == PFPL_OK) st = ensure_hdr(L, s, count);
     if (st != PFPL_OK) return st;
     // every header in one round trip (n and dtype size each output)

@@ -41,6 +41,9 @@ constexpr int kTpUnrollD = PFPL_TP_UNROLL_D;
 #ifndef PFPL_DEC_IO_NS
 #define PFPL_DEC_IO_NS 1024       // the IO warp runs up to 8 chunks ahead: poll rarely
 #endif
+#ifndef PFPL_DEC_LANE_ARRIVE
+#define PFPL_DEC_LANE_ARRIVE 1    // every IO lane arrives on full[] (else lane 0 after __syncwarp)
+#endif
 constexpr int NQD = 8;                 // chunks in flight per CTA (payload queue depth)
 #ifndef PFPL_DEC_RING
 #define PFPL_DEC_RING 24576
@@ -62,7 +65,6 @@ struct DecShared {
     unsigned long long wtot[4];        // per-warp totals of the delta scan
     DecEntry q[NQD];
     unsigned long long full[NQD], empty[NQD];
-    uint32_t tail;                     // ring bytes released by the compute warps (monotone)
     uint32_t sel[16];                  // PRMT selector spreading popc(n) packed bytes to mask n
     uint32_t selr[16];                 // same, unset bits repeating the previous byte (carry = 4)
     unsigned long long vacc[8];        // verify mode: the CTA's metric accumulators (layout of p.vm)
@@ -307,10 +309,9 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         g_pfpl_wd = p.wd;
         if (smem_u32(smem) & 1023u) __trap();
         for (int k = 0; k < NQD; ++k) {
-            mbar_init(smem_u32(&S.full[k]), 1);
+            mbar_init(smem_u32(&S.full[k]), PFPL_DEC_LANE_ARRIVE ? 32 : 1);   // IO lanes (+ the bulk bytes)
             mbar_init(smem_u32(&S.empty[k]), 1);
         }
-        S.tail = 0;
         fence_barrier_init();
     }
     if (tid < 16) {
@@ -340,7 +341,7 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         // offsets are known up front (size_scan_kernel), so no ticket atomics sit on
         // the IO warp's critical path, and the next chunk's table entries are loaded
         // one iteration ahead
-        uint32_t head = 0;
+        uint32_t head = 0, rel = 0;     // ring: next free byte / released up to (monotone)
         const uint64_t G = gridDim.x;
         uint64_t c = blockIdx.x;
         uint32_t size_n = 0;
@@ -350,10 +351,9 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             const int slot = k % NQD;
             if (c >= C) {
                 mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
-                if (lane == 0) {
-                    S.q[slot].c = c;
-                    mbar_arrive(smem_u32(&S.full[slot]));
-                }
+                if (lane == 0) S.q[slot].c = c;
+                __syncwarp();
+                if (PFPL_DEC_LANE_ARRIVE || lane == 0) mbar_arrive(smem_u32(&S.full[slot]));
                 break;
             }
             // d1: chunk offset from the size-table prefix sum (size_scan_kernel)
@@ -370,29 +370,30 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             const uint32_t R = bad ? 16u : ((delta + size + 15u) & ~15u) + 16u;
             const uint32_t head0 = head;
             if (head % RING + R > (uint32_t)RING) head += RING - head % RING;   // never wrap a slice
-            // live bytes are [tail, head0): free if empty or span <= RING
-            auto full = [&]() {
-                const uint32_t t = *(volatile uint32_t*)&S.tail;
-                return t != head0 && head + R - t > (uint32_t)RING;
-            };
-            if (full()) {
-                const uint64_t t0 = globaltimer();
-                uint32_t ns = 64;
-                while (full()) {
-                    if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x23, head);
-                    __nanosleep(ns);
-                    ns = ns < 2048 ? 2 * ns : ns;
-                }
-            }
-            const uint32_t pos = head % RING;
-            head += R;
-            // the IO warp runs up to NQD chunks ahead: waiting here is the common
-            // case, so sleep between polls instead of spinning on the issue port
+            // Ring release protocol (as the encoder's arena): the compute warps arrive on
+            // empty[j % NQD] once chunk j's payload is consumed; the IO warp waits on the
+            // phase of every chunk whose ring bytes it reuses, so each reuse is ordered by
+            // an mbarrier.  First the queue slot (chunk k - NQD), whose ring end `rel`
+            // the IO warp recorded itself; then, if the slice still does not fit (live
+            // bytes [rel, head0) plus the slice span more than RING, and the ring is not
+            // empty), the chunks after it, oldest first.  The IO warp runs up to NQD
+            // chunks ahead: waiting is the common case, so it sleeps between polls.
 #if PFPL_DEC_IO_HINT
             mbar_wait_wd(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21);
 #else
             mbar_wait_sleep(smem_u32(&S.empty[slot]), ((k / NQD) & 1u) ^ 1u, 0x21, PFPL_DEC_IO_NS);
 #endif
+            if (k >= (uint32_t)NQD) rel = __shfl_sync(PFPL_FULL, S.q[slot].rend, 0);
+            auto fits = [&](uint32_t r) { return r == head0 || head + R - r <= (uint32_t)RING; };
+            if (!fits(rel)) {
+                for (uint32_t j = k >= (uint32_t)NQD ? k - NQD + 1 : 0; j < k; ++j) {
+                    mbar_wait_sleep(smem_u32(&S.empty[j % NQD]), (j / NQD) & 1u, 0x23, 64);
+                    rel = __shfl_sync(PFPL_FULL, S.q[j % NQD].rend, 0);
+                    if (fits(rel)) break;
+                }
+            }
+            const uint32_t pos = head % RING;
+            head += R;
             // bulk copy of the aligned superset, never past the last 16-byte
             // boundary of the stream; the remainder by the lanes
             const uint8_t* a0 = g - delta;
@@ -417,10 +418,11 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 if (bulk) {
                     mbar_arrive_tx(smem_u32(&S.full[slot]), bulk);
                     bulk_g2s(smem_u32(stg), a0, bulk, smem_u32(&S.full[slot]));
-                } else {
-                    mbar_arrive(smem_u32(&S.full[slot]));
                 }
             }
+            __syncwarp();
+            if (PFPL_DEC_LANE_ARRIVE ? (lane != 0 || !bulk) : (lane == 0 && !bulk))
+                mbar_arrive(smem_u32(&S.full[slot]));
         }
         return;
     }
@@ -442,11 +444,8 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
         const uint8_t* pay = ring + md.pos + md.delta;
         uint8_t* const dstc = (uint8_t*)p.out + c * (uint64_t)kChunkBytes;
-        auto release = [&]() {
-            if (tid == 0) {
-                *(volatile uint32_t*)&S.tail = md.rend;
-                mbar_arrive(smem_u32(&S.empty[slot]));
-            }
+        auto release = [&]() {          // after a CTA barrier: every read of the payload is done
+            if (tid == 0) mbar_arrive(smem_u32(&S.empty[slot]));
         };
         if (md.bad) {
             named_sync(1, NTC);
@@ -472,14 +471,25 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             continue;
         }
         // ---- levels 4 -> 3 -> 2, derived by every warp (no barrier) ----
-        const uint32_t M4 = (uint32_t)pay[0] | ((uint32_t)pay[1] << 8) | ((uint32_t)pay[2] << 16) |
-                            ((uint32_t)pay[3] << 24);
+        // Corrupt-stream safety: every level's section must fit in
+        // the stored size BEFORE it is read, so a bad bitmap can never steer a read past
+        // the payload's ring slice.  A level that does not fit is treated as empty (no
+        // reads) and the chunk is reported as corrupt; the checks are CTA-uniform (every
+        // warp derives the same counts from the same bytes).
+        uint32_t M4 = (uint32_t)pay[0] | ((uint32_t)pay[1] << 8) | ((uint32_t)pay[2] << 16) |
+                      ((uint32_t)pay[3] << 24);
+        bool fits = 4u + (uint32_t)__popc(M4) <= md.size;
+        if (!fits) M4 = 0u;
         const uint32_t n4 = __popc(M4);
         const uint8_t* z4 = pay + 4;
         const uint32_t c4 = __popc(M4 & (lane == 31 ? 0xFFFFFFFFu : ((2u << lane) - 1u)));
-        const uint32_t m3 = c4 ? z4[c4 - 1] : 0u;              // M3 byte `lane`
-        const uint32_t cnt3 = __popc(m3);
-        const uint32_t inc3 = warp_incl_scan(cnt3, lane);
+        uint32_t m3 = c4 ? z4[c4 - 1] : 0u;                     // M3 byte `lane`
+        uint32_t cnt3 = __popc(m3);
+        uint32_t inc3 = warp_incl_scan(cnt3, lane);
+        if (4u + n4 + __shfl_sync(PFPL_FULL, inc3, 31) > md.size) {
+            fits = false;
+            m3 = cnt3 = inc3 = 0u;
+        }
         const uint32_t n3 = __shfl_sync(PFPL_FULL, inc3, 31);
         const uint8_t* z3 = z4 + n4;
         uint32_t m2lo = 0, m2hi = 0;                            // M2 bytes 8*lane .. 8*lane+7
@@ -509,8 +519,12 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             if (j < 4) m2lo |= bv << (8 * j); else m2hi |= bv << (8 * (j - 4));
         }
 #endif
-        const uint32_t pc2 = __popc(m2lo) + __popc(m2hi);
-        const uint32_t inc2 = warp_incl_scan(pc2, lane);
+        uint32_t pc2 = __popc(m2lo) + __popc(m2hi);
+        uint32_t inc2 = warp_incl_scan(pc2, lane);
+        if (4u + n4 + n3 + __shfl_sync(PFPL_FULL, inc2, 31) > md.size) {
+            fits = false;
+            m2lo = m2hi = pc2 = inc2 = 0u;
+        }
         const uint32_t n2 = __shfl_sync(PFPL_FULL, inc2, 31);
         const uint8_t* z2 = z3 + n3;
         // ---- level 2 -> M1: thread t owns M1 bytes [NB2*t, NB2*t + NB2) ----
@@ -623,7 +637,8 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
             n1 = tot_l + tot_h;
         }
         const uint8_t* z1 = z2 + n2;
-        const bool consistent = 4 + n4 + n3 + n2 + n1 == md.size;
+        const bool consistent = fits && 4 + n4 + n3 + n2 + n1 == md.size;
+        if (!consistent) P = 0;           // no Z1 reads: the gather offsets are not trusted
         uint32_t lo[32], hi[32];
         PFPL_DEC_TIER(dec1_gather, lo, hi, z1, lane, nb, ex, offl, offh, S.sel);
 

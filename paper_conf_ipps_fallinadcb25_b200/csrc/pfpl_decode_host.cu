@@ -28,6 +28,7 @@ int decode_grid(int dtype, int mode, bool ms, uint64_t C) {
         cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, DEC_SMEM);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, dec_threads(dtype), DEC_SMEM);
         g = sms * (per > 0 ? per : 1);
+        if (g > grid_limit()) g = grid_limit();
     }
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
 }

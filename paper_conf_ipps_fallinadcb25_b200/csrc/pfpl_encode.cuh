@@ -62,9 +62,24 @@ constexpr int kTpUnroll = PFPL_TP_UNROLL;
 #ifndef PFPL_TIER4
 #define PFPL_TIER4 0        // P <= 4 uses the 8-plane tier: less hot code (+7% NYX)
 #endif
-#ifndef PFPL_LB_WIDE
-#define PFPL_LB_WIDE 1        // wider windows measured slower (more L2 loads): profiles/r01_tuning.md
+#ifndef PFPL_LANE_ARRIVE
+#define PFPL_LANE_ARRIVE 0    // compute lanes arrive on mq_full one by one (else lane 0 after __syncwarp)
 #endif
+#ifndef PFPL_LANE_ARRIVE_IO
+#define PFPL_LANE_ARRIVE_IO 1 // IO lanes arrive on mq_empty one by one
+#endif
+// arrive on an IO-queue barrier after this lane's own shared-memory accesses (LANES:
+// each lane is its own release, as compute-sanitizer racecheck models it; 32 arrivals)
+// or after the warp's (lane 0, behind __syncwarp; 1 arrival)
+template <bool LANES>
+__device__ __forceinline__ void q_arrive(uint32_t bar, int lane) {
+    if (LANES) {
+        mbar_arrive(bar);
+    } else {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(bar);
+    }
+}
 #ifndef PFPL_LB_NS
 #define PFPL_LB_NS 1500
 #endif
@@ -81,7 +96,7 @@ struct EncShared {
     uint8_t m2[256];
     uint8_t wcnt[128];               // per-warp per-plane Z1 counts, [warp * B + bit]
     uint32_t scan2[4];               // level-2 warp totals
-    uint32_t head, tail;
+    uint32_t head, rel;                // arena: next free byte / released up to (monotone counters)
     unsigned long long in_c[NIN];
     QEntry q[NQ];
     unsigned long long full[NIN], mq_full[NQ], mq_empty[NQ];
@@ -120,6 +135,7 @@ static __device__ void write_header(uint8_t* out, const EncParams& p, const QCon
     put_u64(out + 40, (uint64_t)kChunkBytes);
 }
 
+// [stage] byte scatter (Z1/Z2/Z3 stores)
 // scatter the bytes of w whose marker (0x01 per byte in hh) is set to z[o...]
 __device__ __forceinline__ uint32_t scatter_word(uint8_t* z, uint32_t o, uint32_t w, uint32_t hh) {
     const uint32_t incl = hh * 0x01010101u;
@@ -138,6 +154,7 @@ __device__ __forceinline__ void scatter_marked(uint8_t* z, uint32_t o, uint32_t 
     if (H & 0x80000000u) z[o + (rk >> 24)] = (uint8_t)(w >> 24);
 }
 
+// [stage] IO warp: copy-out
 // copy len bytes from shared memory to global memory, any alignment on either
 // side: 16-byte aligned stores for the body (coalesced even for
 // unaligned compressed data), byte stores for the head and the tail.  Reads up
@@ -170,6 +187,7 @@ void warp_copy_s2g(uint8_t* o, const uint8_t* src, uint32_t len, int lane) {
     }
 }
 
+// [stage] arena allocation
 // ---------------------------------------------------------------------------
 // bit shuffle + level-1 zero-byte elimination for one chunk.
 // KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
@@ -177,10 +195,6 @@ void warp_copy_s2g(uint8_t* o, const uint8_t* src, uint32_t len, int lane) {
 // position is plane p = B-1-b_j, byte p*CW/8 + 4*tid (reading R13).
 // Z1 (plane-major, non-zero bytes in order) goes to the chunk's arena slice.
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t ld_volatile_u32(const uint32_t* p) {
-    return *(const volatile uint32_t*)p;
-}
-
 // Arena slice for a chunk with n1 Z1 bytes: every compute warp derives the same
 // position from S.head (advanced by warp 0 only after the Z1 scatter) and waits
 // only if the IO warp lags by more than the arena's capacity.
@@ -194,50 +208,38 @@ __device__ __forceinline__ uint32_t zroom(uint32_t n1) { return min(2048u, (uint
 __device__ __forceinline__ uint32_t slice_bytes(uint32_t n1, uint32_t n2) {
     return a16(n1) + a16(PRE3 + min(n2, zroom(n1)));
 }
-#ifndef PFPL_ARENA_WAIT_NOINLINE
-#define PFPL_ARENA_WAIT_NOINLINE 0
-#endif
-// out-of-line arena wait: until tail == head0 (arena empty) or tail >= need
-static __device__ __noinline__ void arena_wait(const uint32_t* tail, uint32_t head0, uint32_t need,
-                                               uint32_t head) {
-    const uint64_t t0 = globaltimer();
-    for (;;) {
-        const uint32_t t = ld_volatile_u32(tail);
-        if (t == head0 || (int32_t)(t - need) >= 0) return;
-        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x13, head);
-        __nanosleep(64);
-    }
-}
-
+// Arena release protocol: the IO warp arrives on mq_empty[j % NQ] once it has read
+// (copied out) chunk j's slice; a compute warp that needs arena bytes still held by
+// chunk j waits on that barrier phase itself before writing them, so every reuse of
+// arena bytes is ordered by an mbarrier (release/acquire in the PTX memory model, and
+// visible to compute-sanitizer racecheck).  S.rel = end (monotone byte counter) of
+// chunk it-1-NQ's slice, recorded by the duty warp of iteration it-1 right after its
+// own wait on that chunk (published by this iteration's first CTA barrier).  Queue
+// entries of chunks it-NQ .. it-1 are intact here: the duty warp overwrites chunk
+// it-NQ's only after the third barrier.  The parity wait on chunk j cannot alias: slot
+// j % NQ completes again only for chunk j + NQ >= it, which is not yet pushed.
 template <int ARENA>
-__device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, int lane) {
+__device__ __forceinline__ uint32_t slice_start(const EncShared& S, uint32_t n1, uint32_t it) {
     const uint32_t R = a16(n1) + a16(PRE3 + zroom(n1));     // worst case
     const uint32_t head0 = S.head;
     uint32_t head = head0;
     const uint32_t p0 = head % ARENA;
     if (p0 + R > (uint32_t)ARENA) head += ARENA - p0;      // a slice never wraps
-    // live bytes are [tail, head0); the new slice [head, head+R) is free when the
-    // arena is empty or the live range plus the slice spans at most ARENA bytes
-    // (the gap skipped to avoid wrapping is never released by itself)
-    auto full = [&]() {
-        const uint32_t t = ld_volatile_u32(&S.tail);
-        return t != head0 && head + R - t > (uint32_t)ARENA;
-    };
-#if PFPL_ARENA_WAIT_NOINLINE
-    if (lane == 0 && full()) arena_wait(&S.tail, head0, head + R - (uint32_t)ARENA, head);
-#else
-    if (lane == 0 && full()) {
-        const uint64_t t0 = globaltimer();
-        while (full()) {
-            if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x13, head);
-            __nanosleep(64);
+    // the new slice [head, head+R) is free when every byte before rel is released and
+    // the live range [rel, head0) plus the slice spans at most ARENA bytes, or when the
+    // arena is empty (rel == head0; the gap skipped to avoid wrapping is never
+    // released by itself)
+    auto fits = [&](uint32_t rel) { return rel == head0 || head + R - rel <= (uint32_t)ARENA; };
+    if (!fits(S.rel)) {
+        for (uint32_t j = it - min(it, (uint32_t)NQ); j < it; ++j) {    // oldest first
+            mbar_wait_wd(smem_u32(&S.mq_empty[j % NQ]), (j / NQ) & 1u, 0x13);
+            if (fits(S.q[j % NQ].rend)) break;
         }
     }
-#endif
-    __syncwarp();
     return head;                                            // monotone byte counter
 }
 
+// [stage] level 1: plane counts + scans
 // ---- level-1 phase A: transpose in place, per-plane counts, packed warp scans.
 // KL planes from the low 32 bits of the residuals, KH from the high 32 (f64).
 // Plane word j holds bit b_j of the thread's 32 residuals (b_j = j, or 32+j-KL).
@@ -272,6 +274,7 @@ __device__ __forceinline__ void rze1_count(uint32_t (&lo)[32], uint32_t (&hi)[32
     }
 }
 
+// [stage] level 1: Z1/M1 scatter
 // ---- level-1 phase B: scatter the non-zero bytes of this thread's plane words
 // to Z1 (plane-major order, R13) and its M1 nibbles; offl/offh = this warp's
 // Z1 offset of the segment of bit `lane` / `32+lane`.
@@ -299,6 +302,47 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
     }
 }
 
+// [stage] IO warp: look-back
+// Decoupled look-back (Merrill-Garland) over descriptors hi, hi-1, ..., lo,
+// nearest first, in 32-wide windows (lane l reads descriptor top - l).  rd(idx, &flag)
+// returns the value of descriptor idx and its flag (LB_P inclusive prefix, LB_A
+// aggregate, 0 not yet published).  Returns the sum of the values from the nearest
+// inclusive prefix up to hi and sets *found, or the sum over all of lo..hi if none of
+// them is an inclusive prefix.  Chunks handed out in the same "round" are processed
+// concurrently by the other CTAs' IO warps, so the nearest inclusive prefix is
+// typically one round (~#CTAs chunks) back.  A window is re-read (sleeping between
+// polls, so polling costs the compute warps almost no issue slots) until every
+// descriptor it needs is published.
+template <typename RD>
+__device__ __forceinline__ uint64_t lookback(RD rd, int64_t hi, int64_t lo, int lane, bool* found,
+                                             uint32_t site) {
+    uint64_t acc = 0;
+    const uint64_t t0 = globaltimer();
+    for (int64_t top = hi; top >= lo;) {
+        const int64_t idx = top - lane;
+        const bool valid = idx >= lo;
+        uint32_t flag = 0;
+        const uint64_t v = valid ? rd(idx, flag) : 0ull;
+        const uint32_t pm = __ballot_sync(PFPL_FULL, valid && flag == (uint32_t)LB_P);
+        const uint32_t nr = __ballot_sync(PFPL_FULL, valid && flag == 0u);
+        const uint32_t need = pm ? ((pm & (0u - pm)) << 1) - 1u : PFPL_FULL;
+        if (nr & need) {
+            if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(site, (uint32_t)top);
+            __nanosleep(PFPL_LB_NS);
+            continue;
+        }
+        acc += warp_sum64((valid && ((need >> lane) & 1u)) ? v : 0ull);
+        if (pm) {
+            *found = true;
+            return acc;
+        }
+        top -= 32;
+    }
+    *found = false;
+    return acc;
+}
+
+// [stage] misc (tier dispatch, stats)
 #define PFPL_TIER_DISPATCH(FN, ...)                                                     \
     do {                                                                                \
         if (P == 0) FN<T, 0, 0>(__VA_ARGS__);                                           \
@@ -329,6 +373,7 @@ __device__ __forceinline__ bool is_bin_word(typename Tr<T>::W w, typename Tr<T>:
     return (W)(w - qbias) < LIM;
 }
 
+// [stage] kernel setup + tickets
 template <typename T, int MODE, bool MSR>
 __global__ void __launch_bounds__(Tr<T>::NT + 32, EncCfg<T>::MINB)
 encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
@@ -366,11 +411,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         if (smem_u32(smem) & 1023u) __trap();       // TMA SWIZZLE_128B needs 1024-byte alignment
         for (int s = 0; s < NIN; ++s) mbar_init(smem_u32(&S.full[s]), 1);
         for (int k = 0; k < NQ; ++k) {
-            mbar_init(smem_u32(&S.mq_full[k]), NWC);     // every compute warp arrives
-            mbar_init(smem_u32(&S.mq_empty[k]), 1);
+            mbar_init(smem_u32(&S.mq_full[k]), (PFPL_LANE_ARRIVE ? 32 : 1) * NWC);  // compute lanes/warps
+            mbar_init(smem_u32(&S.mq_empty[k]), PFPL_LANE_ARRIVE_IO ? 32 : 1);     // IO lanes/warp
         }
         S.head = 0;
-        S.tail = 0;
+        S.rel = 0;
         fence_barrier_init();
         prefetch_tmap(&tmap);
     }
@@ -381,6 +426,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     }
 
     if (warp == NWC) {
+// [stage] IO warp: queue
         // =========================== IO warp ===========================
         const uint64_t EP = (uint64_t)p.epoch << 48;
         for (uint32_t k = 0;; ++k) {
@@ -391,63 +437,30 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const uint64_t c = e.c;
             const uint32_t stored = e.stored, start = e.start;
             const bool israw = e.raw != 0;
+// [stage] IO warp: look-back
             // ---- decoupled look-back ----
             uint64_t excl = 0;
             if (c > 0) {
-                // windows of 32*LBW predecessors, lane l reads chunks look-LBW*l-j
-                // (j < LBW, nearest first).  Chunks handed out in the same "round" are
-                // processed concurrently by the other CTAs' IO warps, so the nearest
-                // inclusive prefix is typically one round (~#CTAs chunks) back: wide
-                // windows walk it in a few load latencies.  A window is re-read (after
-                // a short sleep, so polling costs the compute warps almost no issue
-                // slots) until every chunk up to the first inclusive prefix has published.
-                constexpr int LBW = PFPL_LB_WIDE;
-                int64_t look = (int64_t)c - 1;
-                const uint64_t t0 = globaltimer();
-                for (;;) {
-                    uint64_t d[LBW];
-                    const int64_t idx0 = look - LBW * lane;
-#pragma unroll
-                    for (int j = 0; j < LBW; ++j) d[j] = idx0 - j >= 0 ? ld_relaxed(&p.status[idx0 - j]) : 0ull;
-                    int jp = LBW;                 // nearest inclusive prefix in this lane
-                    bool nrl = false;             // a not-yet-published chunk before it
-                    uint64_t sl = 0;
-#pragma unroll
-                    for (int j = LBW - 1; j >= 0; --j) {
-                        uint32_t flag;
-                        uint64_t val;
-                        if (idx0 - j < 0) { flag = (uint32_t)LB_P; val = 0; }        // before chunk 0: prefix 0
-                        else {
-                            flag = ((uint32_t)(d[j] >> 48) == p.epoch) ? (uint32_t)((d[j] >> 46) & 3u) : 0u;
-                            val = d[j] & LB_VAL;
-                        }
-                        if (flag == LB_P) { jp = j; sl = val; nrl = false; }
-                        else { sl += val; nrl = nrl || flag == 0u; }
-                    }
-                    const uint32_t pm = __ballot_sync(PFPL_FULL, jp < LBW);
-                    const uint32_t nr = __ballot_sync(PFPL_FULL, nrl);
-                    const uint32_t need = pm ? ((pm & (0u - pm)) << 1) - 1u : PFPL_FULL;
-                    if (nr & need) {
-                        // a predecessor is still being encoded (typically ~1 chunk time):
-                        // the IO warp's latency is hidden by the arena, so poll rarely
-                        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x12, (uint32_t)look);
-                        __nanosleep(PFPL_LB_NS);
-                        continue;
-                    }
-                    if (pm) {
-                        const int first = __ffs(pm) - 1;
-                        excl += warp_sum64(lane <= first ? sl : 0ull);
-                        break;
-                    }
-                    excl += warp_sum64(sl);
-                    look -= 32 * LBW;
-                }
+                // chunk descriptors: [63:48] epoch | [47:46] flag | [45:0] value
+                auto rd_chunk = [&](int64_t i, uint32_t& flag) -> uint64_t {
+                    const uint64_t d = ld_relaxed(&p.status[i]);
+                    flag = ((uint32_t)(d >> 48) == p.epoch) ? (uint32_t)((d >> 46) & 3u) : 0u;
+                    return d & LB_VAL;
+                };
+                bool found = false;
+                excl = lookback(rd_chunk, (int64_t)c - 1, 0, lane, &found, 0x12);
                 if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + stored));
             }
+// [stage] IO warp: table + copy
             const uint64_t dst = p.payload_off + excl;
             if (lane == 0) {
                 p.table[c] = stored;
-                if (c == C - 1) p.result[0] = dst + stored;
+                if (c == C - 1) {
+                    // stream bytes, and the status word of pfpl_compress_async (pfpl.h):
+                    // offsets are monotone, so the last chunk's end is the stream's end
+                    p.result[0] = dst + stored;
+                    if (dst + stored > p.cap) ((int*)p.result)[2] = -3;     // PFPL_ERR_CAPACITY
+                }
                 if (c == 0 && p.write_header) write_header(p.out, p, qc);
             }
             if (dst + stored <= p.cap) {
@@ -467,15 +480,12 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     warp_copy_s2g(p.out + dst + e.plen, arena + e.z1, stored - e.plen, lane);
                 }
             }
-            __syncwarp();
-            if (lane == 0) {
-                *(volatile uint32_t*)&S.tail = e.rend;     // release the arena slice
-                mbar_arrive(smem_u32(&S.mq_empty[slot]));
-            }
+            q_arrive<PFPL_LANE_ARRIVE_IO>(smem_u32(&S.mq_empty[slot]), lane);   // reads of the slice and entry are done
         }
         return;
     }
 
+// [stage] compute: stage wait + M1 zero
     // ============================ compute warps ============================
     QF<T> q;
     q.load(qc);
@@ -498,6 +508,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         for (int i = 0; i < 2048 / 16 / NTC; ++i)
             ((uint4*)m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
 
+// [stage] quantize + delta (loop)
         // ---- quantize + verify, delta, residual code ----
         uint32_t lo[32], hi[32];
         W orv = 0;
@@ -651,12 +662,14 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 add_raw(nraw);
             }
         }
+// [stage] compute: active planes
         // this warp's active planes (warp-uniform tier; other warps may differ)
         const uint32_t ol = __reduce_or_sync(PFPL_FULL, (uint32_t)orv);
         const uint32_t oh = sizeof(W) == 8 ? __reduce_or_sync(PFPL_FULL, (uint32_t)((uint64_t)orv >> 32)) : 0u;
         const uint64_t wor = ((uint64_t)oh << 32) | ol;
         const int P = wor ? 64 - __clzll((long long)wor) : 0;
 
+// [stage] level 1: plane counts + scans
         // ---- bit shuffle + level-1 zero elimination ----
         uint32_t ex[16];
         PFPL_TIER_DISPATCH(rze1_count, lo, hi, S, lane, warp, wor, ex);
@@ -669,6 +682,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             next = atomicAdd(p.ticket, 1ull);
             issue(s, t);
         }
+// [stage] level 1: offsets + arena
         // Z1 offsets of this warp's segments: planes in decreasing bit order,
         // then warps (lane l owns bit l and 32+l)
         uint32_t offl, offh, n1, head;
@@ -694,13 +708,15 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             offl = tot_h + sl - tl + myl;
             offh = sh - th + myh;
             n1 = tot_l + tot_h;
-            head = slice_start<ARENA>(S, n1, lane);
+            head = slice_start<ARENA>(S, n1, it);
         }
         uint8_t* const z1 = arena + head % ARENA;
+// [stage] level 1: Z1/M1 scatter
         PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
         named_sync(1, NTC);    // Z1 and M1 complete
         uint8_t* const z2 = z1 + a16(n1) + PRE3;
 
+// [stage] level 2
         // ---- level 2: repeated-byte elimination of M1 (2048 B -> M2 + Z2), P:131 ----
         const int slot = it % NQ;
         {
@@ -744,13 +760,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 for (int i = 0; i < NWD2; ++i) o = scatter_word(z2, o, w2[i], h2[i]);
             }
 
+// [stage] levels 3-4 + hand-off
             // ---- levels 3 and 4 on the 256-byte M2, size, raw decision,
             // aggregate, hand-off: one duty warp, rotating so no warp is always late ----
             if (warp != (int)(it % NWC)) {
                 // this warp's Z2 bytes are written: release them to the IO warp (the
                 // entry's phase completes only with the duty warp's arrival)
-                __syncwarp();
-                if (lane == 0) mbar_arrive(smem_u32(&S.mq_full[slot]));
+                q_arrive<PFPL_LANE_ARRIVE>(smem_u32(&S.mq_full[slot]), lane);
                 continue;
             }
             const uint2 v = ((const uint2*)S.m2)[lane];
@@ -777,12 +793,12 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const bool israw = size >= rawb;
             if (israw && lane == 0 && p.stats) atomicAdd(&p.stats[1], 1ull);
             const uint32_t stored = israw ? rawb : size;
-            __syncwarp();
             if (lane == 0) {
                 const uint64_t EP = (uint64_t)p.epoch << 48;
                 st_relaxed(&p.status[c], EP | ((c == 0 ? LB_P : LB_A) << 46) | stored);
                 mbar_wait_wd(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u, 0x15);
                 QEntry& e = S.q[slot];
+                if (it >= NQ) S.rel = e.rend;       // chunk it-NQ's slice is released
                 e.c = c;
                 e.stored = stored;
                 e.raw = israw ? 1u : 0u;
@@ -790,19 +806,22 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 e.plen = 4 + n4 + n3 + n2;
                 e.z1 = head % ARENA;
                 e.rend = head + slice_bytes(n1, n2);
-                mbar_arrive(smem_u32(&S.mq_full[slot]));
             }
+            __syncwarp();
+            q_arrive<PFPL_LANE_ARRIVE>(smem_u32(&S.mq_full[slot]), lane);
         }
     }
+// [stage] kernel exit
     // end of work: tell the IO warp (queue position `it` gets a terminal entry;
     // all compute warps leave at the same `it` and each arrives once)
-    if (lane == 0) {
+    {
         const int slot = it % NQ;
         if (tid == 0) {
             mbar_wait_wd(smem_u32(&S.mq_empty[slot]), ((it / NQ) & 1u) ^ 1u, 0x16);
             S.q[slot].c = ~0ull;
         }
-        mbar_arrive(smem_u32(&S.mq_full[slot]));
+        __syncwarp();
+        q_arrive<PFPL_LANE_ARRIVE>(smem_u32(&S.mq_full[slot]), lane);
     }
 }
 

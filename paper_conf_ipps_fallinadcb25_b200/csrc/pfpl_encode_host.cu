@@ -39,6 +39,7 @@ int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
         prepare_enc(fn, dtype);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, enc_threads(dtype), enc_smem(dtype));
         g = sms * (per > 0 ? per : 1);
+        if (g > grid_limit()) g = grid_limit();
     }
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
 }

@@ -33,7 +33,7 @@ struct EncParams {
     uint64_t cap;            // capacity of out (bytes)
     uint32_t* table;         // size table (local slice)
     uint64_t payload_off;    // payload start relative to out
-    unsigned long long* status;   // look-back descriptors [C]
+    unsigned long long* status;   // look-back descriptors, one per chunk [C]
     unsigned long long* ticket;   // monotone ticket counter
     uint64_t ticket_base;
     uint32_t epoch;
@@ -94,6 +94,10 @@ cudaError_t launch_noa_derive(int dtype, const double* mnmx, double eps, uint32_
 cudaError_t launch_header_only(uint8_t* out, uint64_t n, int dtype, int bound, double eps,
                                const QConst qc, const QConst* qc_dev, uint64_t* result,
                                cudaStream_t s);
+// test knob: PFPL_GRID_LIMIT=k caps the persistent encoder/decoder grids at k CTAs, so
+// small inputs exercise the many-chunks-per-CTA paths (arena and ring wrap-around)
+// quickly, e.g. under compute-sanitizer.  Unset (the default) = full occupancy.
+int grid_limit();
 int encode_grid(int dtype, int mode, bool ms, uint64_t C);
 int encode_stages();
 int decode_grid(int dtype, int mode, bool ms, uint64_t C);
@@ -103,6 +107,10 @@ int decode_tickets_per_cta();
 float log2p_host_f32(float a);
 double log2p_host_f64(double a);
 
+// the host-side argument checks of pfpl_compress_async (pfpl_batch.cu validates every
+// field with it before anything is enqueued)
+int check_compress_args(const void* in, uint64_t n, int dtype, int bound, double eps,
+                        unsigned opts, const void* out, uint64_t cap);
 // records e as the last CUDA error (pfpl_last_cuda_error) and returns PFPL_ERR_CUDA
 int record_cuda_error(int e);
 // free the host-pipeline (pfpl_pipeline.cu) and batch-lane (pfpl_batch.cu) caches of device dev

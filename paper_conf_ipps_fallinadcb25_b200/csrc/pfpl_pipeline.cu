@@ -32,6 +32,7 @@ constexpr uint64_t kDefaultSegChunks = 2048;   // 32 MiB of input per segment
 // Creating streams and mapping 256 MiB of buffers on every call costs more
 // than the transfers themselves (measured: 14 GB/s vs 51 GB/s sequential).
 struct Pipe {
+    std::mutex mu;                  // held for a whole call: one user of the buffers at a time
     cudaStream_t s = nullptr;       // caller's compute stream
     cudaStream_t h2d = nullptr, d2h = nullptr;
     cudaEvent_t in_ready[2] = {}, in_free[2] = {}, out_free[2] = {};
@@ -91,9 +92,12 @@ struct Pipe {
 std::mutex g_pipe_mu;
 std::map<std::pair<int, void*>, Pipe*> g_pipes;
 
-// drains the pipe's streams when a call leaves, on every path
+// owns the pipe for one call (two host threads passing the same stream are
+// serialised instead of sharing its buffers and events); drains the pipe's
+// streams when the call leaves, on every path, before releasing it
 struct PipeUse {
     Pipe* p = nullptr;
+    std::unique_lock<std::mutex> lk;
     ~PipeUse() {
         if (p) p->drain();
     }
@@ -110,6 +114,7 @@ cudaError_t get_pipe(cudaStream_t cs, uint64_t in_bytes, uint64_t out_bytes, Pip
         if (!slot) slot = new Pipe();
         p = slot;
     }
+    use->lk = std::unique_lock<std::mutex>(p->mu);
     use->p = p;
     return p->ensure(cs, in_bytes, out_bytes);
 }
@@ -154,7 +159,10 @@ int pfpl_compress_host(const void* in_host, uint64_t n, int dtype, int bound, do
     const uint64_t ts = tsz_of(dtype);
     const uint64_t cw = kChunkBytes / ts;
     const uint64_t C = (n + cw - 1) / cw;
-    const uint64_t S = seg_chunks ? seg_chunks : kDefaultSegChunks;
+    // S in [1, max(C, 1)]: a larger request means one segment (and keeps S*cw,
+    // k*S*kChunkBytes and the segment count free of overflow)
+    uint64_t S = seg_chunks ? seg_chunks : kDefaultSegChunks;
+    if (S > C) S = C ? C : 1;
     const uint64_t cap = *out_bytes;
     const uint64_t pay_base = kHeaderBytes + 4 * C;
     if (cap < pay_base) return PFPL_ERR_CAPACITY;
@@ -284,29 +292,40 @@ int pfpl_decompress_host(const void* in_host, uint64_t in_bytes, void* out_host,
     const uint32_t* table = (const uint32_t*)(src + kHeaderBytes);   // may be unaligned
     const uint8_t* payload = src + kHeaderBytes + 4 * C;
     const uint64_t pay_bytes = in_bytes - kHeaderBytes - 4 * C;
-    const uint64_t S = seg_chunks ? seg_chunks : kDefaultSegChunks;
-    const uint64_t nseg = (C + S - 1) / S;
-    // segment payload offsets: host prefix sum of the size table
-    uint64_t* seg_off = new uint64_t[nseg + 1];
-    uint32_t* tab = new uint32_t[C ? C : 1];
-    if (C) memcpy(tab, table, 4 * C);
-    uint64_t acc = 0, seg_max = 0;
-    for (uint64_t k = 0; k < nseg; ++k) {
-        seg_off[k] = acc;
-        const uint64_t c1 = (k + 1) * S < C ? (k + 1) * S : C;
-        for (uint64_t c = k * S; c < c1; ++c) acc += tab[c];
-        if (acc - seg_off[k] > seg_max) seg_max = acc - seg_off[k];
+    if (C == 0) {                       // header only: nothing may follow it
+        if (in_bytes != kHeaderBytes) return PFPL_ERR_CORRUPT;
+        *out_bytes = 0;
+        return PFPL_OK;
     }
-    seg_off[nseg] = acc;
+    uint64_t S = seg_chunks ? seg_chunks : kDefaultSegChunks;
+    if (S > C) S = C;
+    const uint64_t nseg = (C + S - 1) / S;
+    // segment payload offsets: host prefix sum of the size table.  Every
+    // entry is validated here, with the rules of the device path (a chunk holds at
+    // most its raw bytes; a compressed chunk at least the 4-byte M4; the sizes sum
+    // to exactly the payload), so a corrupt table is rejected before any device
+    // buffer is sized from it.
+    uint64_t* seg_off = new uint64_t[nseg + 1];
+    uint32_t* tab = new uint32_t[C];
+    memcpy(tab, table, 4 * C);
     struct Free {
         uint64_t* a; uint32_t* b;
         ~Free() { delete[] a; delete[] b; }
     } fr{seg_off, tab};
-    if (acc > pay_bytes) return PFPL_ERR_CORRUPT;
-    if (C == 0) {
-        *out_bytes = 0;
-        return PFPL_OK;
+    uint64_t acc = 0, seg_max = 0;
+    for (uint64_t k = 0; k < nseg; ++k) {
+        seg_off[k] = acc;
+        const uint64_t c1 = (k + 1) * S < C ? (k + 1) * S : C;
+        for (uint64_t c = k * S; c < c1; ++c) {
+            const uint64_t m = c + 1 < C ? cw : n - c * cw;
+            const uint64_t rawb = m * ts;
+            if (tab[c] > rawb || (tab[c] < 4 && tab[c] != rawb)) return PFPL_ERR_CORRUPT;
+            acc += tab[c];
+        }
+        if (acc - seg_off[k] > seg_max) seg_max = acc - seg_off[k];
     }
+    seg_off[nseg] = acc;
+    if (acc != pay_bytes) return PFPL_ERR_CORRUPT;
     cudaStream_t cs = (cudaStream_t)stream;
     const uint64_t seg_out = (C < S ? C : S) * kChunkBytes;
     PipeUse use;

@@ -61,8 +61,11 @@ CONFIGS = {
                            A=10.0, tau=1e-4, zero_frac=0.05),
     "miranda": FieldSpec("Miranda-shaped 256x384x384 f64", (256, 384, 384), "f64", 6,
                          A=1.0, tau=1e-6, offset=2.0),
+    # configs[4]: A recalibrated in round 2 so the f32 ABS 1E-3 ratio is ~19.6 (oracle on
+    # rows 0/300/700), inside the 20 +- 5 band of DESIGN.md 6 (A=0.02 gave ~90: the
+    # 4x finer grid makes the same modes 4x smoother per step)
     "big16g": FieldSpec("16 GiB f32 field 1024x2048x2048", (1024, 2048, 2048), "f32", 7,
-                        A=0.02, tau=1e-3),
+                        A=0.4, tau=1e-3),
 }
 
 

@@ -52,16 +52,17 @@ SIZES = [1, 31, 32, 33, 4095, 4096, 4097, 3 * 4096 + 17, 20000]
 
 @pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
 @pytest.mark.parametrize("dt", [np.float32, np.float64])
-def test_small_fields_all_sizes(pk, orc, bound, dt):
+@pytest.mark.parametrize("eps", [1e-2, 1e-3])
+def test_small_fields_all_sizes(pk, orc, bound, dt, eps):
     for n in SIZES:
         spec = synth.FieldSpec("t", (n,), "f32" if dt == np.float32 else "f64", 3, A=0.5, tau=0.01)
         x = synth.generate(spec).numpy()
-        _check(pk, orc, x, bound, 1e-3)
+        _check(pk, orc, x, bound, eps)
 
 
 @pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
 @pytest.mark.parametrize("dt", [np.float32, np.float64])
-@pytest.mark.parametrize("eps", [1e-1, 1e-4, 0.37])
+@pytest.mark.parametrize("eps", [1e-1, 1e-2, 1e-4, 0.37])
 def test_adversarial(pk, orc, bound, dt, eps):
     x = synth.adversarial_f32() if dt == np.float32 else synth.adversarial_f64()
     _check(pk, orc, x, bound, eps)
@@ -98,7 +99,8 @@ def test_empty(pk, orc):
 
 CONFIGS = [("cesm", "abs", 1e-3), ("hurricane", "rel", 1e-3), ("miranda", "abs", 1e-4),
            ("miranda", "rel", 1e-4), ("miranda", "noa", 1e-4), ("nyx", "abs", 1e-3),
-           ("nyx", "noa", 1e-3)]
+           ("nyx", "noa", 1e-3), ("nyx_rough", "abs", 1e-3), ("cesm", "abs", 1e-2),
+           ("hurricane", "rel", 1e-2), ("miranda", "noa", 1e-2)]
 
 
 @pytest.mark.parametrize("name,bound,eps", CONFIGS)
