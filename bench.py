@@ -156,6 +156,36 @@ def _time_oracle(x, bound, eps, threads, seconds):
     return tc, td, s, reps
 
 
+def _time_cpu_codec(x, s_oracle, bound, eps, cores, seconds):
+    """The multi-core CPU production codec (libpfpl_cpu.so) on the same
+    sample: all host threads and one thread; its stream must equal the oracle's."""
+    import numpy as np
+    from paper_conf_ipps_fallinadcb25_b200 import cpu
+    out = np.empty(cpu.lib().pfpl_cpu_max_compressed_bytes(x.size, 0 if x.dtype == np.float32 else 1), np.uint8)
+    y = np.empty_like(x)
+    res = {"kind": "PFPL CPU codec (OpenMP, AVX2; P:139-168)", "cores": cores,
+           "identical_to_oracle_stream": bytes(cpu.compress(x, bound, eps, out=out)) == s_oracle}
+    for label, nt in (("all_threads", cores), ("single_thread", 1)):
+        s = cpu.compress(x, bound, eps, nthreads=nt, out=out)
+        nb = s.size
+        cpu.decompress(out[:nb], nthreads=nt, out=y)
+        reps = 0
+        t0 = time.perf_counter()
+        while reps < 3 or (time.perf_counter() - t0 < seconds / 4 and reps < 200):
+            cpu.compress(x, bound, eps, nthreads=nt, out=out)
+            reps += 1
+        tc = (time.perf_counter() - t0) / reps
+        reps_d = 0
+        t0 = time.perf_counter()
+        while reps_d < 3 or (time.perf_counter() - t0 < seconds / 4 and reps_d < 200):
+            cpu.decompress(out[:nb], nthreads=nt, out=y)
+            reps_d += 1
+        td = (time.perf_counter() - t0) / reps_d
+        res[label] = {"compress_gbs": x.nbytes / tc / 1e9, "decompress_gbs": x.nbytes / td / 1e9,
+                      "threads": nt, "reps": [reps, reps_d]}
+    return res
+
+
 def cpu_baseline(spec, bound, eps, seconds):
     """The oracle as it stands (plain C, chunks over host threads) on a bounded
     sample of the same workload (the first rows of the field), on the SAME bytes
@@ -171,8 +201,9 @@ def cpu_baseline(spec, bound, eps, seconds):
     # single thread on a quarter of the same sample (whole rows), so the run stays bounded
     x1 = x[:max(inner, (x.size // 4) // inner * inner)]
     tc1, td1, _, reps1 = _time_oracle(x1, bound, eps, 1, 0.4 * seconds)
+    cpu_codec = _time_cpu_codec(x, s, bound, eps, cores, 0.5 * seconds)
     return {"value": x.nbytes / tc / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
-            "cpu_model": cpu_model(),
+            "cpu_model": cpu_model(), "cpu_codec": cpu_codec,
             "sample": f"first {rows} of {spec.shape[0]} rows ({x.nbytes / 1e6:.1f} MB), "
                       f"{reps} reps, OpenMP over chunks on {cores} threads",
             "decompress_gbs": x.nbytes / td / 1e9, "ratio": x.nbytes / len(s),

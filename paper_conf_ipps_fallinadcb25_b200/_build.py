@@ -93,6 +93,23 @@ def build(force: bool = False, verbose: bool = False, jobs: int = os.cpu_count()
     return lib
 
 
+CPU_SRC = os.path.join(PKG, "cpu", "pfpl_cpu.c")
+CPU_LIB = os.path.join(PKG, "libpfpl_cpu.so")
+# the multi-core CPU codec: x86-64-v3 (AVX2, BMI2) + OpenMP; IEEE-strict
+# floating point (no contraction) so its streams are bit-identical to the GPU's
+CPU_FLAGS = ["-O3", "-march=x86-64-v3", "-std=c11", "-fPIC", "-shared", "-fopenmp",
+             "-ffp-contract=off", "-fno-fast-math", "-Wall", "-Wno-unused-parameter"]
+
+
+def build_cpu(force: bool = False) -> str:
+    deps = [CPU_SRC, os.path.join(ROOT, "include", "pfpl_cpu.h")]
+    if force or not os.path.exists(CPU_LIB) or any(os.path.getmtime(d) > os.path.getmtime(CPU_LIB) for d in deps):
+        tmp = CPU_LIB + ".tmp"
+        subprocess.run(["gcc", *CPU_FLAGS, CPU_SRC, "-o", tmp, "-lm"], check=True)
+        os.replace(tmp, CPU_LIB)
+    return CPU_LIB
+
+
 if __name__ == "__main__":
     import sys
     if len(sys.argv) > 2:      # _build.py OUT.so -DFLAG ...   (tuning variants)

@@ -75,7 +75,7 @@ def test_product_never_imports_oracle():
                         assert all(not a.name.startswith("oracle") for a in node.names), f
                     if isinstance(node, ast.ImportFrom):
                         assert not (node.module or "").startswith("oracle"), f
-            if f.endswith((".cu", ".cuh", ".h")):
+            if f.endswith((".cu", ".cuh", ".h", ".c")):
                 assert "oracle" not in open(os.path.join(dirpath, f)).read().lower(), f
 
 
@@ -89,3 +89,17 @@ def test_batch_and_host_bindings_need_no_gpu_for_empty_and_reject_cuda_only_args
         pk.compress_host(torch.zeros(8, 2).t(), "abs", 1e-3)     # non-contiguous host tensor
     with pytest.raises(pk.PFPLError):
         pk.compress_batch([torch.zeros(8)], "abs", 1e-3)       # host tensor where CUDA is required
+
+
+def test_cpu_codec_exports_every_declared_symbol():
+    """libpfpl_cpu.so exports every function of include/pfpl_cpu.h."""
+    import ctypes
+    from paper_conf_ipps_fallinadcb25_b200 import _build
+    path = _build.build_cpu()
+    src = re.sub(r"/\*.*?\*/", "", open(os.path.join(ROOT, "include", "pfpl_cpu.h")).read(), flags=re.S)
+    names = sorted(set(re.findall(r"\b(pfpl_cpu_[a-z_0-9]+)\s*\(", src)))
+    assert len(names) == 4
+    L = ctypes.CDLL(path)
+    for n in names:
+        assert hasattr(L, n), n
+    assert L.pfpl_cpu_max_compressed_bytes(4096, 0) == 48 + 4 + 16384

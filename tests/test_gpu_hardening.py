@@ -162,3 +162,20 @@ def test_full_size_incompressible_stream(pk, orc, dt):
     assert len(s_gpu) == 48 + 4 * C + x.nbytes
     y = pk.decompress(torch.frombuffer(bytearray(s_cpu), dtype=torch.uint8).cuda())
     assert torch.equal(y.view(torch.int32), bits)
+
+
+@pytest.mark.parametrize("name,bound,eps", [("nyx", "abs", 1e-3), ("hurricane", "rel", 1e-3),
+                                            ("miranda", "noa", 1e-4)])
+def test_gpu_and_cpu_codec_interchange(pk, name, bound, eps):
+    """P:43 (data compressed on one device, decompressed on another): at full size the
+    GPU library and the multi-core CPU codec (NEXT-2) write the same stream, and each
+    decodes the other's stream to the same values."""
+    from paper_conf_ipps_fallinadcb25_b200 import cpu
+    xd = synth.generate(synth.CONFIGS[name], device="cuda")
+    x = xd.cpu().numpy()
+    s_gpu = pk.compress(xd, bound, eps).cpu().numpy().tobytes()
+    s_cpu = cpu.compress(x, bound, eps)
+    assert s_gpu == s_cpu
+    y_cpu = cpu.decompress(s_gpu)
+    y_gpu = pk.decompress(torch.frombuffer(bytearray(s_cpu), dtype=torch.uint8).cuda()).cpu().numpy()
+    assert np.array_equal(y_cpu.view(np.uint8), y_gpu.view(np.uint8))
