@@ -355,7 +355,8 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     }
     // d1: prefix sum of the stored sizes -> chunk offsets
     CK(launch_size_scan(table_dev, nchunks, nloc, (uint32_t)cw, (uint32_t)tsz(dtype), payload_bytes,
-                        sc->offs, sc->status, sc->epoch, sc->ticket, sc->ticket_val, err_dev, s));
+                        sc->offs, sc->status, sc->epoch, sc->ticket, sc->ticket_val, err_dev,
+                        watchdog_ptr(), s));
     g_launches += 1;
     sc->ticket_val += (uint64_t)scan_grid(nchunks);
     DecParams p;

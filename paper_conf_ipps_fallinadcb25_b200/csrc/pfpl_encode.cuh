@@ -448,7 +448,12 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     return d & LB_VAL;
                 };
                 bool found = false;
+#if defined(PFPL_LB_FAKE)
+                (void)rd_chunk; (void)found;
+                excl = c * 1024u;    // timing experiment only: no look-back (invalid stream)
+#else
                 excl = lookback(rd_chunk, (int64_t)c - 1, 0, lane, &found, 0x12);
+#endif
                 if (lane == 0) st_relaxed(&p.status[c], EP | (LB_P << 46) | (excl + stored));
             }
 // [stage] IO warp: table + copy
@@ -463,7 +468,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 }
                 if (c == 0 && p.write_header) write_header(p.out, p, qc);
             }
+#if defined(PFPL_NO_COPY)
+            if (false) {         // timing experiment only: no copy-out (invalid stream)
+#else
             if (dst + stored <= p.cap) {
+#endif
                 if (israw) {
                     // raw chunk (R17): stage the original bytes in this chunk's
                     // arena slice (always large enough: slice >= payload >= raw bytes)

@@ -84,7 +84,7 @@ cudaError_t launch_size_scan(const uint32_t* table, uint64_t C, uint64_t n, uint
                              uint32_t s_bytes, uint64_t in_bytes, uint64_t* offs,
                              unsigned long long* status, uint32_t epoch,
                              unsigned long long* ticket, uint64_t tbase, int* err,
-                             cudaStream_t s);
+                             unsigned int* wd, cudaStream_t s);
 cudaError_t launch_minmax(int dtype, const void* in, uint64_t n, double* partial,
                           int blocks, cudaStream_t s);
 cudaError_t launch_minmax_final(const double* partial, int blocks, double* mnmx,

@@ -174,12 +174,15 @@ __global__ void __launch_bounds__(SCAN_T) size_scan_kernel(const uint32_t* table
                                                             uint64_t in_bytes, uint64_t* offs,
                                                             unsigned long long* status, uint32_t epoch,
                                                             unsigned long long* ticket, uint64_t tbase,
-                                                            int* err) {
+                                                            int* err, unsigned int* wd) {
     __shared__ unsigned long long sh_tile;
     __shared__ uint64_t wsum[SCAN_T / 32];
     __shared__ uint64_t sh_excl;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0) sh_tile = atomicAdd(ticket, 1ull) - tbase;
+    if (tid == 0) {
+        g_pfpl_wd = wd;
+        sh_tile = atomicAdd(ticket, 1ull) - tbase;
+    }
     __syncthreads();
     const uint64_t t = sh_tile;
     const uint64_t c0 = t * SCAN_TILE + (uint64_t)tid * SCAN_PER;
@@ -225,10 +228,13 @@ __global__ void __launch_bounds__(SCAN_T) size_scan_kernel(const uint32_t* table
                 const int64_t idx = look - lane;
                 uint64_t val = 0, flag = LB_P;
                 if (idx >= 0) {
+                    const uint64_t t0 = globaltimer();
                     for (;;) {
                         const uint64_t d = ld_relaxed(&status[idx]);
                         flag = ((uint32_t)(d >> 48) == epoch) ? ((d >> 46) & 3u) : 0u;
                         if (flag) { val = d & LB_VAL; break; }
+                        // bounded like every spin loop of the library (watchdog -> trap)
+                        if (globaltimer() - t0 > kWatchdogNs) watchdog_fire(0x31, (uint32_t)idx);
                     }
                 }
                 const uint32_t pm = __ballot_sync(PFPL_FULL, flag == LB_P);
@@ -272,9 +278,9 @@ cudaError_t launch_size_scan(const uint32_t* table, uint64_t C, uint64_t n, uint
                              uint32_t s_bytes, uint64_t in_bytes, uint64_t* offs,
                              unsigned long long* status, uint32_t epoch,
                              unsigned long long* ticket, uint64_t tbase, int* err,
-                             cudaStream_t s) {
+                             unsigned int* wd, cudaStream_t s) {
     size_scan_kernel<<<scan_grid(C), SCAN_T, 0, s>>>(table, C, n, cw, s_bytes, in_bytes, offs,
-                                                     status, epoch, ticket, tbase, err);
+                                                     status, epoch, ticket, tbase, err, wd);
     return cudaGetLastError();
 }
 
