@@ -263,8 +263,8 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
     const int grid = encode_grid(dtype, mode, ms, C);
     CK(launch_encode(dtype, mode, ms, p, grid, s));
     g_launches += 1;
-    // each persistent encoder CTA consumes NSTAGE + 1 tickets beyond its chunks
-    sc->ticket_val += C + (uint64_t)grid * (uint64_t)(encode_stages() + 1);
+    // each persistent encoder CTA consumes (stages + 1) tickets per pipeline beyond its chunks
+    sc->ticket_val += C + (uint64_t)grid * (uint64_t)encode_tickets_per_cta(dtype);
     return PFPL_OK;
 }
 

@@ -115,6 +115,8 @@ template <typename T> struct EncCfg {
     static constexpr int SHARED_OFF = ARENA_OFF + ARENA + 64;
     static constexpr int SMEM = SHARED_OFF + (int)sizeof(EncShared);
     static constexpr int MINB = sizeof(T) == 4 ? PFPL_ENC_MINB : PFPL_ENC_MINB64;
+    static constexpr int THREADS = Tr<T>::NT + 32;          // compute warps + the IO warp
+    static constexpr int TICKETS = NIN + 1;                 // tickets a CTA draws beyond its chunks
     static_assert(SMEM <= 233472 / MINB - 1024, "MINB CTAs per SM must fit in shared memory");
     static_assert(DATAB + 16 + ((PRE3 + 15) & ~15) <= ARENA, "the arena must hold a worst-case slice");
 };

@@ -20,7 +20,7 @@ static void* pick_enc(int dtype, int mode, bool ms) {
     return tab[dtype ? 1 : 0][mode & 3](ms);
 }
 
-static int enc_threads(int dtype) { return (dtype == 0 ? Tr<float>::NT : Tr<double>::NT) + 32; }
+static int enc_threads(int dtype) { return dtype == 0 ? EncCfg<float>::THREADS : EncCfg<double>::THREADS; }
 
 static int enc_smem(int dtype) { return dtype == 0 ? EncCfg<float>::SMEM : EncCfg<double>::SMEM; }
 
@@ -44,7 +44,7 @@ int encode_grid(int dtype, int mode, bool ms, uint64_t C) {
     return (int)(C < (uint64_t)g ? C : (uint64_t)g);
 }
 
-int encode_stages() { return NIN; }
+int encode_tickets_per_cta(int dtype) { return dtype == 0 ? EncCfg<float>::TICKETS : EncCfg<double>::TICKETS; }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
                                   const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,

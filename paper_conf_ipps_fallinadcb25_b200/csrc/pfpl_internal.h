@@ -99,7 +99,7 @@ cudaError_t launch_header_only(uint8_t* out, uint64_t n, int dtype, int bound, d
 // quickly, e.g. under compute-sanitizer.  Unset (the default) = full occupancy.
 int grid_limit();
 int encode_grid(int dtype, int mode, bool ms, uint64_t C);
-int encode_stages();
+int encode_tickets_per_cta(int dtype);   // tickets a persistent encoder CTA draws beyond its chunks
 int decode_grid(int dtype, int mode, bool ms, uint64_t C);
 int decode_tickets_per_cta();
 
