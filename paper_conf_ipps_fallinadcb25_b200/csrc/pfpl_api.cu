@@ -158,6 +158,13 @@ int host_qconst(int dtype, int bound, double eps, unsigned opts, QConst* qc, int
         const float w = 2.0f * lw;
         if (!(w > 0.0f) || std::isinf(w)) { qc->flags |= HF_RAWWORDS; *mode = MODE_RAW; return PFPL_OK; }
         qc->a = f2u_h(c); qc->b = f2u_h(w); qc->c = f2u_h(0.5f / lw); qc->qconst = f2u_h(w);
+        // fast-path margin in bin units: |log2p - lg2.approx| <= 3.6e-7 +
+        // 2.4e-7 |L|, the roundings of s (2.4e-7 |L| c), y, the R7 window and pow2p
+        // (<= 2.2e-6 + 7.4e-7 |L| in all, in log2 units), with >= 2.7x headroom
+        const double cinv = 0.5 / (double)lw;
+        const double m1 = cinv * 2e-6, m2 = cinv * 8e-6;
+        qc->m1 = f2u_h(0.0f); qc->m2 = f2u_h(1.0f);          // 1: the fast path never certifies
+        if (m2 < 0.2 && m1 * 128.0 + m2 < 0.25) { qc->m1 = f2u_h((float)m1); qc->m2 = f2u_h((float)m2); }
     } else {
         double c;
         if (eps < 4503599627370496.0) {
@@ -171,6 +178,12 @@ int host_qconst(int dtype, int bound, double eps, unsigned opts, QConst* qc, int
         const double w = 2.0 * lw;
         if (!(w > 0.0) || std::isinf(w)) { qc->flags |= HF_RAWWORDS; *mode = MODE_RAW; return PFPL_OK; }
         qc->a = d2u_h(c); qc->b = d2u_h(w); qc->c = d2u_h(0.5 / lw); qc->qconst = d2u_h(w);
+        // f64 fast path: L from the exact exponent + lg2.approx.f32 of the mantissa (abs
+        // error <= ~4e-7), margin with ~4x headroom
+        const double cinv = 0.5 / lw;
+        const double m1 = cinv * 1e-12, m2 = cinv * 2e-6;
+        qc->m1 = d2u_h(0.0); qc->m2 = d2u_h(1.0);
+        if (m2 < 0.2 && m1 * 1024.0 + m2 < 0.25) { qc->m1 = d2u_h(m1); qc->m2 = d2u_h(m2); }
     }
     return PFPL_OK;
 }

@@ -221,8 +221,11 @@ __device__ __forceinline__ int64_t unzz(uint64_t z) { return (int64_t)((z >> 1) 
 
 template <typename T> struct QF;
 template <> struct QF<float> {
-    float a, b, c;
-    __device__ __forceinline__ void load(const QConst& q) { a = u2f((uint32_t)q.a); b = u2f((uint32_t)q.b); c = u2f((uint32_t)q.c); }
+    float a, b, c, m1, m2;
+    __device__ __forceinline__ void load(const QConst& q) {
+        a = u2f((uint32_t)q.a); b = u2f((uint32_t)q.b); c = u2f((uint32_t)q.c);
+        m1 = u2f((uint32_t)q.m1); m2 = u2f((uint32_t)q.m2);
+    }
     // ABS/NOA: a = eps_eff, b = inv, c = eb2.  Bin = rint(v*inv); decode
     // immediately and keep the bin only if |v - bin*2eps| <= eps (R7);
     // |bin| < 2^22 so the zigzag code stays in the denormal range (R8).
@@ -316,6 +319,36 @@ template <> struct QF<float> {
         }
         return q0 ^ 0xFF800000u;
     }
+    // REL fast path: the bin decision of rel_q taken from lg2.approx when it is certain.
+    // s_exact = fl(log2p(a) * c) and s_fast = fl(lg2.approx(a) * c) differ by less than
+    // margin(L) = m1*|L| + m2 (host: bounds of both log approximations and of the
+    // roundings of s, y = bin*w and the R7 window, with headroom), so when
+    // |s_fast - rint(s_fast)| <= 0.5 - margin, rint(s_exact) = rint(s_fast) = k, and the
+    // reconstruction 2^(k w) lies inside [a/c_lo, a*c_lo] by at least the same margin:
+    // rel_q accepts.  |L| <= 125.5 keeps pow2p away from its inf/0 clamps.  Otherwise
+    // `slow` is set and the caller runs rel_q (same bits either way).
+    __device__ __forceinline__ uint32_t rel_q_fast(float v, bool& slow) const {
+        // branch-free: every quantity is computed, the word is selected at the end
+        const uint32_t u = f2u(v), sign = u >> 31, au = u & 0x7FFFFFFFu;
+        const bool normal = au - 0x00800000u < 0x7F800000u - 0x00800000u;   // finite, not denormal/0
+        float L;
+        asm("lg2.approx.f32 %0, %1;" : "=f"(L) : "f"(u2f(au)));
+        const float s = L * c;
+        const float ts = s + 12582912.0f;
+        const float k = ts - 12582912.0f;
+        const float aL = fabsf(L);
+        // margin test |s - k| <= 0.5 - (m1 |L| + m2) (m2 >= 0.5 disables the path); the
+        // FMA is margin arithmetic only, outside the format's operations
+        const float lim = __fmaf_rn(-m1, aL, 0.5f - m2);
+        const bool certain = (fabsf(s - k) <= lim) & (aL <= 125.5f);
+        // bin word (R10, R11): payload 1 + (zigzag(k) << 1 | sign) = |4k + 1| + sign,
+        // exact as a float for |k| < 2^21; the sign+exponent inversion cancels the NaN tag
+        const uint32_t binw = f2u(fabsf(__fmaf_rn(k, 4.0f, 1.0f)) + 8388608.0f) - 0x4B000000u + sign;
+        const uint32_t lossw = (au > 0x7F800000u ? au : u) ^ 0xFF800000u;
+        const bool bin = normal & certain & (fabsf(k) < 2097152.0f);
+        slow = normal & !certain;
+        return bin ? binw : lossw;
+    }
     __device__ __forceinline__ float rel_dq(uint32_t w) const {
         uint32_t u = w ^ 0xFF800000u;
         if ((u & 0xFF800000u) == 0xFF800000u && (u & 0x007FFFFFu) != 0) {
@@ -327,8 +360,10 @@ template <> struct QF<float> {
     }
 };
 template <> struct QF<double> {
-    double a, b, c;
-    __device__ __forceinline__ void load(const QConst& q) { a = u2d(q.a); b = u2d(q.b); c = u2d(q.c); }
+    double a, b, c, m1, m2;
+    __device__ __forceinline__ void load(const QConst& q) {
+        a = u2d(q.a); b = u2d(q.b); c = u2d(q.c); m1 = u2d(q.m1); m2 = u2d(q.m2);
+    }
     __device__ __forceinline__ uint64_t abs_q(double v) const {
         double s = v * b;
         double t = s + 6755399441055744.0;          // 1.5 * 2^52
@@ -365,6 +400,28 @@ template <> struct QF<double> {
             }
         }
         return q0 ^ 0xFFF0000000000000ull;
+    }
+    // f64 form of QF<float>::rel_q_fast: L = exponent (exact) + lg2.approx.f32 of the
+    // mantissa truncated to binary32; |L| <= 1021.5 keeps pow2p away from its clamps
+    __device__ __forceinline__ uint64_t rel_q_fast(double v, bool& slow) const {
+        const uint64_t u = d2u(v), sign = u >> 63, au = u & 0x7FFFFFFFFFFFFFFFull;
+        const bool normal = au - 0x0010000000000000ull < 0x7FF0000000000000ull - 0x0010000000000000ull;
+        const int e = (int)(au >> 52) - 1023;
+        float lm;
+        asm("lg2.approx.f32 %0, %1;" : "=f"(lm) : "f"(u2f(0x3F800000u | (uint32_t)((au >> 29) & 0x7FFFFFu))));
+        const double L = i2d_small(e) + (double)lm;
+        const double s = L * c;
+        const double ts = s + 6755399441055744.0;
+        const double k = ts - 6755399441055744.0;
+        const double aL = fabs(L);
+        const double lim = __fma_rn(-m1, aL, 0.5 - m2);
+        const bool certain = (fabs(s - k) <= lim) & (aL <= 1021.5);
+        // payload 1 + (zigzag(k) << 1 | sign) = |4k + 1| + sign, exact for |k| < 2^50
+        const uint64_t binw = d2u(fabs(__fma_rn(k, 4.0, 1.0)) + 4503599627370496.0) - 0x4330000000000000ull + sign;
+        const uint64_t lossw = (au > 0x7FF0000000000000ull ? au : u) ^ 0xFFF0000000000000ull;
+        const bool bin = normal & certain & (fabs(k) < 1125899906842624.0);
+        slow = normal & !certain;
+        return bin ? binw : lossw;
     }
     __device__ __forceinline__ double rel_dq(uint64_t w) const {
         uint64_t u = w ^ 0xFFF0000000000000ull;

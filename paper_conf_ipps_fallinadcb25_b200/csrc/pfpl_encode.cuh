@@ -513,11 +513,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         const uint8_t* buf = smem + s * DATAB;
         uint8_t* const m1 = S.m1;
         const uint32_t m = (uint32_t)min((uint64_t)CW, p.n - c * (uint64_t)CW);
-
-        // zero this thread's part of M1
+        if constexpr (MODE != MODE_REL) {
+            // zero this thread's part of M1
 #pragma unroll
-        for (int i = 0; i < 2048 / 16 / NTC; ++i)
-            ((uint4*)m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
+            for (int i = 0; i < 2048 / 16 / NTC; ++i)
+                ((uint4*)m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
+        }
+
 
 // [stage] quantize + delta (loop)
         // ---- quantize + verify, delta, residual code ----
@@ -586,6 +588,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     }
                     __syncwarp();
                     uint32_t nraw = 0;
+                    uint32_t slowm = 0;     // REL: values whose fast-path bin is not certain
 #pragma unroll kTpUnroll
                     for (int i = 0; i < 2 * S_; ++i) {
                         const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
@@ -596,14 +599,72 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         memcpy(x, &v, 16);
 #pragma unroll
                         for (int k = 0; k < 16 / S_; ++k) {
-                            w[k] = quantize_b<T, MODE>(q, x[k], raw);
-                            nraw += is_bin_word<T, MODE>(w[k], (W)qbias, raw) ? 0u : 1u;
+                            if constexpr (MODE == MODE_REL) {
+                                bool sl;
+                                const W fw = q.rel_q_fast(x[k], sl);
+                                // an uncertain value keeps its input bits for the exact pass
+                                W xb;
+                                memcpy(&xb, &x[k], sizeof(W));
+                                w[k] = sl ? xb : fw;
+                                slowm |= (sl ? 1u : 0u) << (i * (16 / S_) + k);
+                                nraw += (sl || is_bin_word<T, MODE>(fw, (W)qbias, raw)) ? 0u : 1u;
+                            } else {
+                                w[k] = quantize_b<T, MODE>(q, x[k], raw);
+                                nraw += is_bin_word<T, MODE>(w[k], (W)qbias, raw) ? 0u : 1u;
+                            }
                         }
                         memcpy(&v, w, 16);
                         *a = v;
                     }
+                    if constexpr (MODE == MODE_REL) {
+                        // the exact quantizer (rel_q, the oracle's arithmetic) for the few
+                        // uncertain values, spread over the warp's lanes: each
+                        // lane lists its values (element id = 32 * lane + j) in this warp's
+                        // share of M1 (zeroed only afterwards), then lane l takes entries
+                        // l, l + 32, ...; above 256 entries every lane does its own
+                        const uint32_t cnt = __popc(slowm);
+                        const uint32_t inc = warp_incl_scan(cnt, lane);
+                        const uint32_t total = __shfl_sync(PFPL_FULL, inc, 31);
+                        auto exact_at = [&](int ol, int j) {
+                            const int i = j / (16 / S_), k = j % (16 / S_);
+                            const int t = 32 * warp + ol;
+                            const int r = sizeof(T) == 4 ? t : 2 * t + (i >> 3);
+                            W* const e = (W*)(wbuf + r * 128 + (((i & 7) ^ (r & 7)) << 4)) + k;
+                            T xv;
+                            memcpy(&xv, e, sizeof(T));
+                            const W wv = quantize_b<T, MODE>(q, xv, raw);
+                            *e = wv;
+                            nraw += is_bin_word<T, MODE>(wv, (W)qbias, raw) ? 0u : 1u;
+                        };
+                        if (total && total <= 256) {
+                            // this warp's own share of M1 (the part its threads zero next)
+                            uint16_t* const list = (uint16_t*)(S.m1 + (2048 / NWC) * warp);
+                            uint32_t o = inc - cnt;
+#pragma unroll 1
+                            for (uint32_t mm = slowm; mm; mm &= mm - 1u) list[o++] = (uint16_t)((lane << 5) | (__ffs(mm) - 1));
+                            __syncwarp();
+#pragma unroll 1
+                            for (uint32_t g = lane; g < total; g += 32) {
+                                const uint32_t id = list[g];
+                                exact_at((int)(id >> 5), (int)(id & 31u));
+                            }
+                            __syncwarp();
+                        } else if (total) {
+#pragma unroll 1
+                            for (uint32_t mm = slowm; mm; mm &= mm - 1u) exact_at(lane, __ffs(mm) - 1);
+                            __syncwarp();
+                        }
+                    }
                     add_raw(nraw);
-                    if (tid > 0) qprev = quantize_b<T, MODE>(q, pv, raw);
+                    if (tid > 0) {
+                        if constexpr (MODE == MODE_REL) {
+                            bool sl;
+                            qprev = q.rel_q_fast(pv, sl);
+                            if (sl) qprev = quantize_b<T, MODE>(q, pv, raw);
+                        } else {
+                            qprev = quantize_b<T, MODE>(q, pv, raw);
+                        }
+                    }
                     fence_proxy_async();      // the stage is refilled by TMA after the next barrier
 #pragma unroll
                     for (int i = 0; i < 2 * S_; ++i) {
@@ -672,6 +733,13 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                 }
                 add_raw(nraw);
             }
+        }
+        // zero this thread's part of M1; REL after its quantizer, which uses this warp's
+        // share as scratch (M1 is written only after the next CTA barrier)
+        if constexpr (MODE == MODE_REL) {
+#pragma unroll
+            for (int i = 0; i < 2048 / 16 / NTC; ++i)
+                ((uint4*)m1)[tid * (2048 / 16 / NTC) + i] = make_uint4(0, 0, 0, 0);
         }
 // [stage] compute: active planes
         // this warp's active planes (warp-uniform tier; other warps may differ)

@@ -23,6 +23,9 @@ struct QConst {
     double range;      // header offset 32 (NOA)
     uint32_t flags;    // header byte 7
     uint32_t pad;
+    // REL encoder fast path: margin(L) = m1*|L| + m2 in bin units, bits of
+    // T; 0 = always the exact path
+    uint64_t m1, m2;
 };
 
 struct EncParams {

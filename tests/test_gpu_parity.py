@@ -334,3 +334,43 @@ def test_full_size_16gib_sampled(pk, orc):
         assert np.array_equal(yc.view(np.uint32), orc.decompress(ref).view(np.uint32)), c
     del x, y, s
     torch.cuda.empty_cache()
+
+
+def _rel_edge_values(orc, dt, eps):
+    """Values within 12 ulps of r_b (1+eps) and r_b / (1+eps) for many bins b (the REL
+    bins' edges, where the exact check decides; R7), plus the largest/smallest
+    exponents (pow2p's clamps) -- the inputs that probe the encoder's REL fast path."""
+    bits = 32 if dt == np.float32 else 64
+    P = orc.params(np.ones(1, dt), "rel", eps)
+    bins = np.concatenate([np.arange(-400, 400, 7), np.arange(2000, 2200, 13),
+                           np.arange(30000, 44000, 997)])
+    zz = np.where(bins >= 0, 2 * bins, -2 * bins - 1).astype(np.int64)
+    mask = 0xFF800000 if bits == 32 else 0xFFF0000000000000
+    words = [((mask | (1 + (int(z) << 1))) ^ mask) for z in zz if (1 + (int(z) << 1)) < (1 << (22 if bits == 32 else 51))]
+    r = orc.dequantize(np.array(words, dtype=np.uint32 if bits == 32 else np.uint64), P).astype(np.float64)
+    r = r[np.isfinite(r) & (r > 0)]
+    with np.errstate(over="ignore"):
+        centers = np.concatenate([(r * (1 + eps)).astype(dt), (r / (1 + eps)).astype(dt)])
+    centers = centers[np.isfinite(centers) & (centers > 0)]
+    vals = [centers]
+    up = down = centers
+    for _ in range(12):
+        up = np.nextafter(up, dt(np.inf))
+        down = np.nextafter(down, dt(0))
+        vals += [up, down]
+    fi = np.finfo(dt)
+    extremes = np.array([fi.max, fi.max / 1.5, fi.tiny, fi.tiny * 1.5, fi.tiny * 3, 2.0 ** (fi.maxexp - 2)], dt)
+    x = np.concatenate(vals + [extremes]).astype(dt)
+    x = np.concatenate([x, -x])
+    return x[np.isfinite(x)]
+
+
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+@pytest.mark.parametrize("eps", [2.0 ** -10, 1e-1, 1e-2, 1e-3, 1e-4, 1e-6])
+def test_rel_bin_edges_and_extremes(pk, orc, dt, eps):
+    """REL parity where the encoder's fast path must defer to the exact quantizer: bin
+    edges (|s - k| close to 1/2) and the exponent extremes (pow2p's inf/0 clamps)."""
+    x = _rel_edge_values(orc, dt, eps)
+    cw = 16384 // np.dtype(dt).itemsize
+    x = np.resize(x, ((x.size + cw - 1) // cw) * cw)     # full chunks: the fast-path layout
+    _check(pk, orc, x, "rel", eps)
