@@ -617,7 +617,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         *a = v;
                     }
                     if constexpr (MODE == MODE_REL) {
-                        // the exact quantizer (rel_q, the oracle's arithmetic) for the few
+                        // the exact quantizer (rel_q, the format's definition) for the few
                         // uncertain values, spread over the warp's lanes: each
                         // lane lists its values (element id = 32 * lane + j) in this warp's
                         // share of M1 (zeroed only afterwards), then lane l takes entries
