@@ -272,6 +272,7 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
     p.wd = watchdog_ptr();
     p.stats = st_cur;
     p.stats_next = st_next;
+    p.nz2 = 0x8000000080000000ull;
     const bool ms = (opts & PFPL_OPT_MS_RESIDUALS) != 0;
     const int grid = encode_grid(dtype, mode, ms, C);
     CK(launch_encode(dtype, mode, ms, p, grid, s));

@@ -203,6 +203,39 @@ __device__ __forceinline__ double pow2p_f64_d(double y) {
     return p * u2d((uint64_t)(ki + 1023) << 52);
 }
 
+// ------------------------------------------------------------------------
+// packed binary32 pairs (FFMA2 / FADD2, sm_100): two IEEE operations per instruction,
+// each lane rounded on its own.  ptxas contracts mul.rn.f32x2 + add.rn.f32x2 into
+// one FFMA2 (a single rounding) even with -fmad=false, so a product is formed as
+// fma(a, b, nz2) with nz2 = (-0, -0) supplied at run time: a*b + (-0) = a*b exactly
+// (also for a*b = -0), and ptxas cannot fold an unknown addend into the next add.
+// ------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t pk(float lo, float hi) {
+    return ((uint64_t)f2u(hi) << 32) | f2u(lo);
+}
+__device__ __forceinline__ float pk_lo(uint64_t x) { return u2f((uint32_t)x); }
+__device__ __forceinline__ float pk_hi(uint64_t x) { return u2f((uint32_t)(x >> 32)); }
+__device__ __forceinline__ uint64_t pk_mul(uint64_t a, uint64_t b, uint64_t nz2) {
+    uint64_t r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(nz2));
+    return r;
+}
+__device__ __forceinline__ uint64_t pk_fma(uint64_t a, uint64_t b, uint64_t c) {   // exact cases only
+    uint64_t r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
+__device__ __forceinline__ uint64_t pk_add(uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ uint64_t pk_sub(uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+
 // predicated select that the compiler cannot turn into a branch
 __device__ __forceinline__ uint32_t selp_u32(uint32_t a, uint32_t b, bool p) {
     uint32_t r;
@@ -274,6 +307,22 @@ template <> struct QF<float> {
         ok = ok && (fabsf(rb) < 4194304.0f) && (diff <= a);
         const float w2 = __fmaf_rn(rb, 2.0f, 0.5f);
         return f2u(fabsf(w2) + 8388607.5f);
+    }
+    // abs_qf on a packed pair (v = values 2i, 2i+1): the same IEEE operations in the same
+    // order, two per instruction (s = v*inv, t = s + 1.5*2^23, rb = t - 1.5*2^23,
+    // vr = rb*eb2, v - vr, and the exact 2*rb + 0.5)
+    __device__ __forceinline__ void abs_qf2(uint64_t v, bool& ok0, bool& ok1, uint32_t& z0, uint32_t& z1,
+                                            uint64_t nz2) const {
+        const uint64_t s = pk_mul(v, pk(b, b), nz2);
+        const uint64_t t = pk_add(s, pk(12582912.0f, 12582912.0f));
+        const uint64_t rb = pk_add(t, pk(-12582912.0f, -12582912.0f));
+        const uint64_t vr = pk_mul(rb, pk(c, c), nz2);
+        const uint64_t d = pk_sub(v, vr);
+        ok0 = ok0 && (fabsf(pk_lo(rb)) < 4194304.0f) && (fabsf(pk_lo(d)) <= a);
+        ok1 = ok1 && (fabsf(pk_hi(rb)) < 4194304.0f) && (fabsf(pk_hi(d)) <= a);
+        const uint64_t w2 = pk_fma(rb, pk(2.0f, 2.0f), pk(0.5f, 0.5f));     // exact for |rb| < 2^22
+        z0 = f2u(fabsf(pk_lo(w2)) + 8388607.5f);
+        z1 = f2u(fabsf(pk_hi(w2)) + 8388607.5f);
     }
     __device__ __forceinline__ float abs_dq(uint32_t w) const {
         return w < 0x00800000u ? __int2float_rn(unzz(w)) * c : u2f(w);

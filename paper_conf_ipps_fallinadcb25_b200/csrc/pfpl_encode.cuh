@@ -80,6 +80,9 @@ __device__ __forceinline__ void q_arrive(uint32_t bar, int lane) {
         if (lane == 0) mbar_arrive(bar);
     }
 }
+#ifndef PFPL_PACKED_Q
+#define PFPL_PACKED_Q 1       // the f32 ABS/NOA fast-path quantizer on FFMA2/FADD2 pairs
+#endif
 #ifndef PFPL_LB_NS
 #define PFPL_LB_NS 1500
 #endif
@@ -550,8 +553,14 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     for (int i = 0; i < 8; ++i) {
                         const uint4 v = *(const uint4*)(buf + tid * 128 + (((i & 7) ^ (tid & 7)) << 4));
                         bool* o = ok + 4 * (i & 1);
+#if PFPL_PACKED_Q
+                        uint32_t z0, z1, z2, z3;
+                        q.abs_qf2(((uint64_t)v.y << 32) | v.x, o[0], o[1], z0, z1, p.nz2);
+                        q.abs_qf2(((uint64_t)v.w << 32) | v.z, o[2], o[3], z2, z3, p.nz2);
+#else
                         const uint32_t z0 = q.abs_qf(u2f(v.x), o[0]), z1 = q.abs_qf(u2f(v.y), o[1]);
                         const uint32_t z2 = q.abs_qf(u2f(v.z), o[2]), z3 = q.abs_qf(u2f(v.w), o[3]);
+#endif
                         const uint32_t r0 = rcode<MSR>(z0 - zp), r1 = rcode<MSR>(z1 - z0);
                         const uint32_t r2 = rcode<MSR>(z2 - z1), r3 = rcode<MSR>(z3 - z2);
                         zp = z3;

@@ -50,6 +50,7 @@ struct EncParams {
     unsigned int* wd;        // watchdog report (mapped host memory) or null
     unsigned long long* stats;       // [0] unquantizable values, [1] raw chunks (this call)
     unsigned long long* stats_next;  // the other slot: zeroed for the next call
+    uint64_t nz2;            // two binary32 -0.0 (0x8000000080000000), opaque to ptxas: see pk_mul
 };
 
 struct DecParams {
