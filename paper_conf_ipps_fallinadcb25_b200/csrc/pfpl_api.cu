@@ -395,6 +395,7 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     p.vbound = bound;
     p.veps = eps_h;
     p.vrange = range_h;
+    p.nz2 = 0x8000000080000000ull;
     const bool ms = (flags & HF_MS) != 0;
     const int grid = decode_grid(dtype, mode, ms, nchunks);
     CK(launch_decode(dtype, mode, ms, p, grid, s));

@@ -710,9 +710,16 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                     W w[16 / S_];
                     T y[16 / S_];
                     memcpy(w, &v, 16);
+                    if constexpr (sizeof(T) == 4 && MODE == MODE_REL) {
+                        const uint64_t y01 = q.rel_dq2((uint32_t)w[0], (uint32_t)w[1], p.nz2);
+                        const uint64_t y23 = q.rel_dq2((uint32_t)w[2], (uint32_t)w[3], p.nz2);
+                        v = make_uint4((uint32_t)y01, (uint32_t)(y01 >> 32), (uint32_t)y23, (uint32_t)(y23 >> 32));
+                        (void)y;
+                    } else {
 #pragma unroll
-                    for (int k = 0; k < 16 / S_; ++k) y[k] = dequantize<T, MODE>(q, w[k], raw);
-                    memcpy(&v, y, 16);
+                        for (int k = 0; k < 16 / S_; ++k) y[k] = dequantize<T, MODE>(q, w[k], raw);
+                        memcpy(&v, y, 16);
+                    }
                     *a = v;
                 }
                 done = true;

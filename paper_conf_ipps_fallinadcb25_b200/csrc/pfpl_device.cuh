@@ -398,6 +398,37 @@ template <> struct QF<float> {
         slow = normal & !certain;
         return bin ? binw : lossw;
     }
+    // rel_dq on a pair of words: the same IEEE operations (bin*w, rint by 1.5*2^23, f, the
+    // degree-7 Horner of pow2p, the power-of-two scale), two per instruction
+    __device__ __forceinline__ uint64_t rel_dq2(uint32_t w0, uint32_t w1, uint64_t nz2) const {
+        const uint32_t u0 = w0 ^ 0xFF800000u, u1 = w1 ^ 0xFF800000u;
+        const uint32_t t0 = (u0 & 0x007FFFFFu) - 1u, t1 = (u1 & 0x007FFFFFu) - 1u;
+        const uint64_t bin = pk(i2f_small(unzz(t0 >> 1)), i2f_small(unzz(t1 >> 1)));   // exact, |bin| < 2^21
+        const uint64_t y = pk_mul(bin, pk(b, b), nz2);
+        const uint64_t tk = pk_add(y, pk(12582912.0f, 12582912.0f));
+        const uint64_t k = pk_add(tk, pk(-12582912.0f, -12582912.0f));
+        const uint64_t f = pk_sub(y, k);
+        uint64_t p = pk(u2f(0x377FE5FEu), u2f(0x377FE5FEu));
+        p = pk_add(pk_mul(p, f, nz2), pk(u2f(0x39218489u), u2f(0x39218489u)));
+        p = pk_add(pk_mul(p, f, nz2), pk(u2f(0x3AAEC3FFu), u2f(0x3AAEC3FFu)));
+        p = pk_add(pk_mul(p, f, nz2), pk(u2f(0x3C1D955Bu), u2f(0x3C1D955Bu)));
+        p = pk_add(pk_mul(p, f, nz2), pk(u2f(0x3D635847u), u2f(0x3D635847u)));
+        p = pk_add(pk_mul(p, f, nz2), pk(u2f(0x3E75FDF0u), u2f(0x3E75FDF0u)));
+        p = pk_add(pk_mul(p, f, nz2), pk(u2f(0x3F317218u), u2f(0x3F317218u)));
+        p = pk_add(pk_mul(p, f, nz2), pk(1.0f, 1.0f));
+        // scale 2^k (k in [-126, 127]; the clamps below replace out-of-range results)
+        const int ki0 = (int)((uint32_t)tk - 0x4B400000u), ki1 = (int)((uint32_t)(tk >> 32) - 0x4B400000u);
+        const int c0 = ki0 < -126 ? -126 : (ki0 > 127 ? 127 : ki0), c1 = ki1 < -126 ? -126 : (ki1 > 127 ? 127 : ki1);
+        const uint64_t mag = pk_mul(p, pk(u2f((uint32_t)(c0 + 127) << 23), u2f((uint32_t)(c1 + 127) << 23)), nz2);
+        auto fin = [&](uint32_t u, uint32_t t, float kf, float m) -> uint32_t {
+            float r = m;
+            if (!(kf <= 127.0f)) r = u2f(0x7F800000u);
+            else if (kf < -126.0f) r = 0.0f;
+            const uint32_t rb = f2u(r) | ((t & 1u) << 31);
+            return ((u & 0xFF800000u) == 0xFF800000u && (u & 0x007FFFFFu) != 0) ? rb : u;
+        };
+        return ((uint64_t)fin(u1, t1, pk_hi(k), pk_hi(mag)) << 32) | fin(u0, t0, pk_lo(k), pk_lo(mag));
+    }
     __device__ __forceinline__ float rel_dq(uint32_t w) const {
         uint32_t u = w ^ 0xFF800000u;
         if ((u & 0xFF800000u) == 0xFF800000u && (u & 0x007FFFFFu) != 0) {

@@ -76,6 +76,7 @@ struct DecParams {
     unsigned long long* vm;
     int vbound;              // bound of the stream (header byte 6)
     double veps, vrange;     // user eps and the NOA range d (header fields)
+    uint64_t nz2;            // two binary32 -0.0, opaque to ptxas (pfpl_device.cuh pk_mul)
 };
 
 // kernel launchers (pfpl_kernels.cu)
