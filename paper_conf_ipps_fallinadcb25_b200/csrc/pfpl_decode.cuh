@@ -51,6 +51,11 @@ constexpr int NQD = 8;                 // chunks in flight per CTA (payload queu
 #ifndef PFPL_DEC_MINB
 #define PFPL_DEC_MINB 5
 #endif
+// f64: 4 CTAs per SM fit 168 registers; REL/NOA gain from a 5th CTA (128 registers,
+// a few spills; Miranda REL +4%, NOA +9%), ABS loses 1.5%
+#ifndef PFPL_DEC_MINB64
+#define PFPL_DEC_MINB64(MODE) ((MODE) == MODE_ABS ? 4 : 5)
+#endif
 constexpr int RING = PFPL_DEC_RING;    // circular payload ring (bytes, multiple of 16)
 
 struct DecEntry {
@@ -292,7 +297,7 @@ struct VerNone {
 };
 
 template <typename T, int MODE, bool MSR, bool VER = false>
-__global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_DEC_MINB : 4)
+__global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_DEC_MINB : PFPL_DEC_MINB64(MODE))
 decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
     constexpr int B = Tr<T>::B, CW = Tr<T>::CW, NTC = Tr<T>::NT, NWC = Tr<T>::NW, S_ = Tr<T>::S;

@@ -33,6 +33,7 @@ PFPL_HD float u2f(uint32_t x) { union { float f; uint32_t u; } v; v.u = x; retur
 PFPL_HD uint64_t d2u(double x) { union { double f; uint64_t u; } v; v.f = x; return v.u; }
 PFPL_HD double u2d(uint64_t x) { union { double f; uint64_t u; } v; v.u = x; return v.f; }
 
+// [stage] quantize (ABS/REL/NOA + verify)
 // ------------------------------------------------------------------------
 // portable log2 / pow2.  Format-version-1 constants: nearest binary32 /
 // binary64 to 2/(k ln 2) (atanh series of log2) and ln2^j/j! (Taylor of 2^f).
@@ -203,6 +204,7 @@ __device__ __forceinline__ double pow2p_f64_d(double y) {
     return p * u2d((uint64_t)(ki + 1023) << 52);
 }
 
+// [stage] quantize (ABS/REL/NOA + verify)
 // ------------------------------------------------------------------------
 // packed binary32 pairs (FFMA2 / FADD2, sm_100): two IEEE operations per instruction,
 // each lane rounded on its own.  ptxas contracts mul.rn.f32x2 + add.rn.f32x2 into
@@ -244,6 +246,7 @@ __device__ __forceinline__ uint32_t selp_u32(uint32_t a, uint32_t b, bool p) {
     return r;
 }
 
+// [stage] quantize (ABS/REL/NOA + verify)
 // ------------------------------------------------------------------------
 // quantizers: value -> word (bin code or raw bits)
 // ------------------------------------------------------------------------
@@ -547,6 +550,7 @@ template <> __device__ __forceinline__ double dequantize<double, MODE_NOA>(const
 template <> __device__ __forceinline__ double dequantize<double, MODE_REL>(const QF<double>& q, uint64_t w, bool) { return q.rel_dq(w); }
 template <> __device__ __forceinline__ double dequantize<double, MODE_RAW>(const QF<double>&, uint64_t w, bool) { return u2d(w); }
 
+// [stage] delta + residual code
 // ------------------------------------------------------------------------
 // residual codes: negabinary (default) or zigzag (flag A1)
 // ------------------------------------------------------------------------
@@ -565,6 +569,7 @@ template <bool MS> __device__ __forceinline__ uint64_t rdecode(uint64_t r) {
               : ((r ^ 0xAAAAAAAAAAAAAAAAull) - 0xAAAAAAAAAAAAAAAAull);
 }
 
+// [stage] bit-plane transpose
 // ------------------------------------------------------------------------
 // bit-plane transpose of 32 words with values < 2^K (K in {4,8,16,32}):
 // out[b] bit j = bit b of in[j].  Pack 32/K elements per word (element j at
@@ -636,6 +641,7 @@ template <int K> __device__ __forceinline__ void transpose_inv(uint32_t (&r)[32]
     }
 }
 
+// [stage] byte masks (zero/repeat elimination)
 // ------------------------------------------------------------------------
 // byte helpers
 // ------------------------------------------------------------------------
@@ -655,6 +661,7 @@ __device__ __forceinline__ uint64_t rankcount(uint32_t H) {
 // gather the low bits of the 4 bytes of h (values 0/1) into a nibble
 __device__ __forceinline__ uint32_t nib(uint32_t h) { return (h * 0x10204080u) >> 28; }
 
+// [stage] warp scans / sums
 // ------------------------------------------------------------------------
 // scans
 // ------------------------------------------------------------------------
@@ -680,6 +687,7 @@ __device__ __forceinline__ uint64_t warp_sum64(uint64_t v) {
     return v;
 }
 
+// [stage] look-back descriptors
 // ------------------------------------------------------------------------
 // look-back descriptors: [63:48] epoch | [47:46] flag | [45:0] value
 // ------------------------------------------------------------------------
@@ -701,6 +709,7 @@ __device__ __forceinline__ uint4 ldg_nc_v4(const void* p) {
     return v;
 }
 
+// [stage] mbarrier / TMA / watchdog waits
 // ------------------------------------------------------------------------
 // sm_90+/sm_100 asynchronous primitives: mbarrier, TMA, named barriers
 // ------------------------------------------------------------------------

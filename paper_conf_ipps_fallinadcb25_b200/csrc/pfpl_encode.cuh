@@ -62,6 +62,10 @@ constexpr int kTpUnroll = PFPL_TP_UNROLL;
 #ifndef PFPL_TIER4
 #define PFPL_TIER4 0        // P <= 4 uses the 8-plane tier: less hot code (+7% NYX)
 #endif
+#ifndef PFPL_UNIFIED_L1
+#define PFPL_UNIFIED_L1 -1    // level-1 code: 1 one windowed path for all tiers, 0 one copy per
+                              // tier, -1 per instantiation (see the kernel)
+#endif
 #ifndef PFPL_LANE_ARRIVE
 #define PFPL_LANE_ARRIVE 0    // compute lanes arrive on mq_full one by one (else lane 0 after __syncwarp)
 #endif
@@ -307,6 +311,84 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
     }
 }
 
+// [stage] level 1: plane counts + scans
+// ---- level 1 with one copy of the count/scatter code for every tier: only the
+// transpose is specialised on the tier (P <= 8, 16, 32 planes; f64 adds the high
+// half), which leaves plane word b of the thread's residuals in lo[b] / hi[b - 32]
+// for every tier.  Counts and scatter then walk windows of 8 planes guarded by the
+// active-plane count P (planes >= P are zero in the whole warp), so a CTA whose
+// warps run different tiers executes one code path: the tiered copies overflowed
+// the 32 KB instruction cache on rough data (ncu: 31% no_instruction stalls).
+template <typename T>
+__device__ __forceinline__ void rze1_transpose(uint32_t (&lo)[32], uint32_t (&hi)[32], int P) {
+    if (P == 0) {
+    } else if (Tr<T>::B == 32 || P <= 32) {
+        if (P <= 8 && PFPL_MIN_TIER <= 8) transpose_fwd<8>(lo);
+        else if (P <= 16 && PFPL_MIN_TIER <= 16) transpose_fwd<16>(lo);
+        else transpose_fwd<32>(lo);
+    } else {
+        transpose_fwd<32>(lo);
+        if (P <= 40) transpose_fwd<8>(hi);
+        else if (P <= 48) transpose_fwd<16>(hi);
+        else transpose_fwd<32>(hi);
+    }
+}
+template <typename T>
+__device__ __forceinline__ void rze1_count_w(const uint32_t (&lo)[32], const uint32_t (&hi)[32], EncShared& S,
+                                             int lane, int warp, uint64_t wor, int P, uint32_t (&ex)[16]) {
+    constexpr int B = Tr<T>::B;
+#pragma unroll
+    for (int w8 = 0; w8 < B / 8; ++w8) {
+        if (P > 8 * w8) {
+#pragma unroll
+            for (int gg = 0; gg < 2; ++gg) {
+                const int b0 = 8 * w8 + 4 * gg;
+                uint32_t inc = 0, v = 0;
+                if (wor & (0xFull << b0)) {          // skip groups empty in this whole warp
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const uint32_t w = b0 + i < 32 ? lo[(b0 + i) & 31] : hi[(b0 + i) & 31];
+                        v = __byte_perm(v, (uint32_t)(rankcount(nzmark(w)) >> 32),
+                                        i == 0 ? 0x3214 : i == 1 ? 0x3240 : i == 2 ? 0x3410 : 0x4210);
+                    }
+                    inc = warp_incl_scan(v, lane);
+                }
+                ex[b0 / 4] = inc - v;
+                if (lane == 31) *(uint32_t*)&S.wcnt[warp * B + b0] = inc;
+            }
+        } else if (lane == 31) {
+            *(uint32_t*)&S.wcnt[warp * B + 8 * w8] = 0u;
+            *(uint32_t*)&S.wcnt[warp * B + 8 * w8 + 4] = 0u;
+        }
+    }
+}
+// [stage] level 1: Z1/M1 scatter
+template <typename T>
+__device__ __forceinline__ void rze1_scatter_w(const uint32_t (&lo)[32], const uint32_t (&hi)[32],
+                                               uint8_t* z1, uint8_t* m1, int tid, int lane, uint64_t wor,
+                                               int P, const uint32_t (&ex)[16], uint32_t offl, uint32_t offh) {
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW;
+#pragma unroll
+    for (int w8 = 0; w8 < B / 8; ++w8) {
+        if (P <= 8 * w8) break;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const int b = 8 * w8 + i;
+            const uint32_t w = b < 32 ? lo[b & 31] : hi[b & 31];
+            if (!((wor >> b) & 1u)) continue;                       // plane empty in this warp
+            if (!__any_sync(PFPL_FULL, w != 0)) continue;
+            const int pl = B - 1 - b;
+            const uint32_t H = nzmark(w);
+            const uint32_t o = __shfl_sync(PFPL_FULL, b < 32 ? offl : offh, b & 31) +
+                               __byte_perm(ex[b / 4], 0, 0x4440 + (b % 4));
+            scatter_marked(z1, o, w, H);
+            const uint32_t nb = nib(H >> 7);
+            const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
+            if (!(lane & 1)) m1[pl * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
+        }
+    }
+}
+
 // [stage] IO warp: look-back
 // Decoupled look-back (Merrill-Garland) over descriptors hi, hi-1, ..., lo,
 // nearest first, in 32-wide windows (lane l reads descriptor top - l).  rd(idx, &flag)
@@ -354,7 +436,7 @@ __device__ __forceinline__ uint64_t lookback(RD rd, int64_t hi, int64_t lo, int 
         else if (B == 32 || P <= 32) {                                                  \
             if (PFPL_TIER4 && P <= 4) FN<T, 4, 0>(__VA_ARGS__);                         \
             else if (P <= 8 && PFPL_MIN_TIER <= 8) FN<T, 8, 0>(__VA_ARGS__);            \
-            else if (P <= 16) FN<T, 16, 0>(__VA_ARGS__);                                \
+            else if (P <= 16 && PFPL_MIN_TIER <= 16) FN<T, 16, 0>(__VA_ARGS__);         \
             else FN<T, 32, 0>(__VA_ARGS__);                                             \
         } else {                                                                        \
             if (P <= 36) FN<T, 32, 4>(__VA_ARGS__);                                     \
@@ -760,7 +842,19 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
 // [stage] level 1: plane counts + scans
         // ---- bit shuffle + level-1 zero elimination ----
         uint32_t ex[16];
-        PFPL_TIER_DISPATCH(rze1_count, lo, hi, S, lane, warp, wor, ex);
+        // level-1 code shape (PFPL_UNIFIED_L1): one copy per tier lets the compiler
+        // free the registers of planes above the tier, which the smooth f32 ABS fields
+        // (NYX: +13%) need; the shared windowed path keeps the hot code of the REL / NOA
+        // quantizers and of f64 inside the instruction cache (Miranda f64 +17-25%,
+        // rough f32 +7%; profiles/r02_encoder_budget.md)
+        constexpr bool kUni = PFPL_UNIFIED_L1 == 1 ||
+                              (PFPL_UNIFIED_L1 < 0 && !(sizeof(T) == 4 && (MODE == MODE_ABS || MODE == MODE_RAW)));
+        if constexpr (kUni) {
+            rze1_transpose<T>(lo, hi, P);
+            rze1_count_w<T>(lo, hi, S, lane, warp, wor, P, ex);
+        } else {
+            PFPL_TIER_DISPATCH(rze1_count, lo, hi, S, lane, warp, wor, ex);
+        }
         named_sync(1, NTC);    // counts visible; every row of stage s consumed
         if (tid == 0) {
             // refill stage s with the prefetched ticket; prefetch the next one
@@ -800,7 +894,8 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         }
         uint8_t* const z1 = arena + head % ARENA;
 // [stage] level 1: Z1/M1 scatter
-        PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
+        if constexpr (kUni) rze1_scatter_w<T>(lo, hi, z1, m1, tid, lane, wor, P, ex, offl, offh);
+        else PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
         named_sync(1, NTC);    // Z1 and M1 complete
         uint8_t* const z2 = z1 + a16(n1) + PRE3;
 

@@ -2,7 +2,7 @@
 config on one GPU.  Device time = CUDA events around the async C-ABI calls
 (median of K after W warm-ups; inputs resident in HBM); `api` = the blocking
 pfpl_compress call (adds its host sync + 8-byte D2H).  Prints a markdown table,
-writes gpurun_out/bench_all.json.   usage: bench_all.py [big] [case-filter]"""
+writes gpurun_out/bench_all.json.   usage: bench_all.py [big] [case-filter | name:bound:eps ...]"""
 import json, os, statistics, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -18,7 +18,9 @@ if big:
     CASES = [("big16g", "abs", 1e-3)]
     args = args[1:]
 if args:
-    CASES = [c for c in CASES if any(a in f"{c[0]}_{c[1]}" for a in args)]
+    # "name:bound:eps" adds an ad-hoc case; other args filter the table's cases
+    extra = [(a.split(":")[0], a.split(":")[1], float(a.split(":")[2])) for a in args if a.count(":") == 2]
+    CASES = [c for c in CASES if any(a in f"{c[0]}_{c[1]}" for a in args)] + extra
 K, W = 10, 3
 res = []
 print("| config | bound | MB | ratio | compress GB/s | decompress GB/s | compress roofline | decompress roofline | api compress GB/s |")

@@ -12,18 +12,24 @@ import subprocess
 import sys
 from collections import defaultdict
 
-# (file, first line, last line, stage) -- first match wins; device.cuh helpers
-# are attributed by what they implement
-STAGES = [
-    ("pfpl_device.cuh", 42, 212, "quantize (ABS/REL/NOA + verify)"),
-    ("pfpl_device.cuh", 213, 412, "quantize (ABS/REL/NOA + verify)"),
-    ("pfpl_device.cuh", 413, 430, "delta + residual code"),
-    ("pfpl_device.cuh", 431, 501, "bit-plane transpose"),
-    ("pfpl_device.cuh", 502, 520, "byte masks (zero/repeat elimination)"),
-    ("pfpl_device.cuh", 521, 545, "warp scans / sums"),
-    ("pfpl_device.cuh", 546, 566, "look-back descriptors"),
-    ("pfpl_device.cuh", 567, 710, "mbarrier / TMA / watchdog waits"),
-]
+# device.cuh helpers are attributed by the "// [stage]" section markers of the
+# sources (see stage_map), i.e. by what they implement
+STAGES = []
+
+
+def stage_map():
+    """(file, first line, last line, stage) from the "// [stage] NAME" markers."""
+    import os
+    import re
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    extra = []
+    for fn in ("pfpl_encode.cuh", "pfpl_decode.cuh", "pfpl_device.cuh"):
+        lines = open(os.path.join(root, "paper_conf_ipps_fallinadcb25_b200", "csrc", fn)).read().splitlines()
+        marks = [(i + 1, m.group(1)) for i, l in enumerate(lines) if (m := re.search(r"// \[stage\] (.+)$", l))]
+        for j, (ln, name) in enumerate(marks):
+            end = marks[j + 1][0] - 1 if j + 1 < len(marks) else len(lines)
+            extra.append((fn, ln, end, name))
+    return extra
 
 
 def load(rep, ksub):
@@ -64,18 +70,7 @@ def stage_of(f, ln, extra):
 
 def main():
     rep, ksub, n = sys.argv[1], sys.argv[2], float(sys.argv[3])
-    extra = []
-    # encoder / decoder line map, read from the section markers of the sources
-    import re
-    import os
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    for fn in ("pfpl_encode.cuh", "pfpl_decode.cuh"):
-        p = os.path.join(root, "paper_conf_ipps_fallinadcb25_b200", "csrc", fn)
-        lines = open(p).read().splitlines()
-        marks = [(i + 1, m.group(1)) for i, l in enumerate(lines) if (m := re.search(r"// \[stage\] (.+)$", l))]
-        for j, (ln, name) in enumerate(marks):
-            end = marks[j + 1][0] - 1 if j + 1 < len(marks) else len(lines)
-            extra.append((fn, ln, end, name))
+    extra = stage_map()
     recs = load(rep, ksub)
     tot = sum(v[0] for v in recs.values())
     tst = sum(v[1] for v in recs.values()) or 1
