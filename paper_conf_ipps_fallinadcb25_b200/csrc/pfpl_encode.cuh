@@ -66,6 +66,9 @@ constexpr int kTpUnroll = PFPL_TP_UNROLL;
 #define PFPL_UNIFIED_L1 -1    // level-1 code: 1 one windowed path for all tiers, 0 one copy per
                               // tier, -1 per instantiation (see the kernel)
 #endif
+#ifndef PFPL_STAGED_L1
+#define PFPL_STAGED_L1 1      // REL: level 1 from plane words staged in shared memory
+#endif
 #ifndef PFPL_LANE_ARRIVE
 #define PFPL_LANE_ARRIVE 0    // compute lanes arrive on mq_full one by one (else lane 0 after __syncwarp)
 #endif
@@ -385,6 +388,83 @@ __device__ __forceinline__ void rze1_scatter_w(const uint32_t (&lo)[32], const u
             const uint32_t nb = nib(H >> 7);
             const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
             if (!(lane & 1)) m1[pl * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
+        }
+    }
+}
+
+// [stage] level 1: plane counts + scans
+// ---- staged level 1 (the two-pass REL / f64 quantizers, whose stage rows are
+// already rewritten in place): after the transpose every thread stores its plane
+// words to its own stage rows (group g of 4 planes = one swizzled 16-byte slot),
+// so counts and scatter are rolled loops over plane groups -- ~2 KB of code for
+// every tier and both halves of f64 instead of an unrolled copy per plane -- and
+// the planes need no registers across the CTA barrier.  The stage is refilled by
+// TMA only after the scatter.
+template <typename T>
+__device__ __forceinline__ uint8_t* plane_slot(uint8_t* wbuf, int tid, int g) {
+    const int r = sizeof(T) == 4 ? tid : 2 * tid + (g >> 3);
+    return wbuf + r * 128 + (((g & 7) ^ (r & 7)) << 4);
+}
+// number of non-zero bytes of each of the 4 words, one per byte (each <= 4)
+__device__ __forceinline__ uint32_t nzcount4(const uint4 v) {
+    uint32_t c = (uint32_t)(rankcount(nzmark(v.x)) >> 32);
+    c = __byte_perm(c, (uint32_t)(rankcount(nzmark(v.y)) >> 32), 0x3240);
+    c = __byte_perm(c, (uint32_t)(rankcount(nzmark(v.z)) >> 32), 0x3410);
+    c = __byte_perm(c, (uint32_t)(rankcount(nzmark(v.w)) >> 32), 0x4210);
+    return c;
+}
+template <typename T>
+__device__ __forceinline__ void rze1_stage_planes(const uint32_t (&lo)[32], const uint32_t (&hi)[32],
+                                                  uint8_t* wbuf, int tid, int P) {
+#pragma unroll
+    for (int g = 0; g < Tr<T>::B / 4; ++g) {
+        if (4 * g < P) {
+            const uint32_t* src = g < 8 ? lo + 4 * g : hi + 4 * (g - 8);
+            *(uint4*)plane_slot<T>(wbuf, tid, g) = make_uint4(src[0], src[1], src[2], src[3]);
+        }
+    }
+}
+template <typename T>
+__device__ __forceinline__ void rze1_count_s(uint8_t* wbuf, EncShared& S, int tid, int lane, int warp,
+                                             uint64_t wor, int P) {
+    constexpr int B = Tr<T>::B;
+    const int ng = (P + 3) >> 2;
+#pragma unroll 1
+    for (int g = 0; g < B / 4; ++g) {
+        uint32_t tot = 0;
+        if (g < ng && (wor & (0xFull << (4 * g)))) {        // warp-uniform
+            const uint4 v4 = *(const uint4*)plane_slot<T>(wbuf, tid, g);
+            tot = __reduce_add_sync(PFPL_FULL, nzcount4(v4));  // bytes <= 128: no carries
+        }
+        if (lane == 31) *(uint32_t*)&S.wcnt[warp * B + 4 * g] = tot;
+    }
+}
+// [stage] level 1: Z1/M1 scatter
+template <typename T>
+__device__ __forceinline__ void rze1_scatter_s(uint8_t* wbuf, uint8_t* z1, uint8_t* m1, int tid, int lane,
+                                               uint64_t wor, int P, uint32_t offl, uint32_t offh) {
+    constexpr int B = Tr<T>::B, CW = Tr<T>::CW;
+    const int ng = (P + 3) >> 2;
+#pragma unroll 1
+    for (int g = 0; g < ng; ++g) {
+        if (!(wor & (0xFull << (4 * g)))) continue;          // warp-uniform
+        const uint4 v4 = *(const uint4*)plane_slot<T>(wbuf, tid, g);
+        const uint32_t cnt = nzcount4(v4);
+        const uint32_t ex = warp_incl_scan(cnt, lane) - cnt;
+        const uint32_t w4[4] = {v4.x, v4.y, v4.z, v4.w};
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const int b = 4 * g + i;
+            const uint32_t w = w4[i];
+            if (!((wor >> b) & 1u)) continue;                   // plane empty in this warp
+            if (!__any_sync(PFPL_FULL, w != 0)) continue;
+            const uint32_t H = nzmark(w);
+            const uint32_t o = __shfl_sync(PFPL_FULL, b < 32 ? offl : offh, b & 31) +
+                               __byte_perm(ex, 0, 0x4440 + i);
+            scatter_marked(z1, o, w, H);
+            const uint32_t nb = nib(H >> 7);
+            const uint32_t nb2 = __shfl_xor_sync(PFPL_FULL, nb, 1);
+            if (!(lane & 1)) m1[(B - 1 - b) * (CW / 64) + (tid >> 1)] = (uint8_t)(nb | (nb2 << 4));
         }
     }
 }
@@ -849,14 +929,22 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         // rough f32 +7%; profiles/r02_encoder_budget.md)
         constexpr bool kUni = PFPL_UNIFIED_L1 == 1 ||
                               (PFPL_UNIFIED_L1 < 0 && !(sizeof(T) == 4 && (MODE == MODE_ABS || MODE == MODE_RAW)));
-        if constexpr (kUni) {
+        // staged level 1 for REL (two-pass quantizer): Hurricane +18%, Miranda f64 +5%;
+        // f64 ABS/NOA lose 6-8% to the later stage refill and keep the windowed path
+        constexpr bool kStg = PFPL_STAGED_L1 && MODE == MODE_REL;
+        uint8_t* const sbuf = smem + s * DATAB;
+        if constexpr (kStg) {
+            rze1_transpose<T>(lo, hi, P);
+            rze1_stage_planes<T>(lo, hi, sbuf, tid, P);
+            rze1_count_s<T>(sbuf, S, tid, lane, warp, wor, P);
+        } else if constexpr (kUni) {
             rze1_transpose<T>(lo, hi, P);
             rze1_count_w<T>(lo, hi, S, lane, warp, wor, P, ex);
         } else {
             PFPL_TIER_DISPATCH(rze1_count, lo, hi, S, lane, warp, wor, ex);
         }
         named_sync(1, NTC);    // counts visible; every row of stage s consumed
-        if (tid == 0) {
+        if (!kStg && tid == 0) {
             // refill stage s with the prefetched ticket; prefetch the next one
             // (the raw ticket is kept: subtracting the base here would wait for the
             // atomic's round trip right before the next barrier)
@@ -894,9 +982,20 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         }
         uint8_t* const z1 = arena + head % ARENA;
 // [stage] level 1: Z1/M1 scatter
-        if constexpr (kUni) rze1_scatter_w<T>(lo, hi, z1, m1, tid, lane, wor, P, ex, offl, offh);
-        else PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
+        if constexpr (kStg) {
+            rze1_scatter_s<T>(sbuf, z1, m1, tid, lane, wor, P, offl, offh);
+            fence_proxy_async();      // the planes' stage is refilled by TMA after the barrier
+        } else if constexpr (kUni) {
+            rze1_scatter_w<T>(lo, hi, z1, m1, tid, lane, wor, P, ex, offl, offh);
+        } else {
+            PFPL_TIER_DISPATCH(rze1_scatter, lo, hi, z1, m1, tid, lane, wor, ex, offl, offh);
+        }
         named_sync(1, NTC);    // Z1 and M1 complete
+        if (kStg && tid == 0) {
+            const unsigned long long t = next - p.ticket_base;
+            next = atomicAdd(p.ticket, 1ull);
+            issue(s, t);
+        }
         uint8_t* const z2 = z1 + a16(n1) + PRE3;
 
 // [stage] level 2
