@@ -28,6 +28,9 @@ namespace pfpl {
 #ifndef PFPL_TP_UNROLL_D
 #define PFPL_TP_UNROLL_D 1
 #endif
+#ifndef PFPL_DQ64_BF
+#define PFPL_DQ64_BF 1        // f64 REL dequantize without branches (interleaved Horner chains)
+#endif
 constexpr int kTpUnrollD = PFPL_TP_UNROLL_D;
 #ifndef PFPL_DEC_LUT
 #define PFPL_DEC_LUT 1     // PRMT-selector gathers (+8% NYX, +17% rough decode)
@@ -720,6 +723,10 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                         const uint64_t y23 = q.rel_dq2((uint32_t)w[2], (uint32_t)w[3], p.nz2);
                         v = make_uint4((uint32_t)y01, (uint32_t)(y01 >> 32), (uint32_t)y23, (uint32_t)(y23 >> 32));
                         (void)y;
+                    } else if constexpr (sizeof(T) == 8 && MODE == MODE_REL && PFPL_DQ64_BF) {
+                        y[0] = q.rel_dq_bf((uint64_t)w[0]);
+                        y[1] = q.rel_dq_bf((uint64_t)w[1]);
+                        memcpy(&v, y, 16);
                     } else {
 #pragma unroll
                         for (int k = 0; k < 16 / S_; ++k) y[k] = dequantize<T, MODE>(q, w[k], raw);

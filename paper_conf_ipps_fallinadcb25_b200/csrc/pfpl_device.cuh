@@ -506,6 +506,38 @@ template <> struct QF<double> {
         slow = normal & !certain;
         return bin ? binw : lossw;
     }
+    // rel_dq without branches (the same IEEE operations; non-bin words compute a
+    // discarded value), so the decoder can interleave the 26-operation Horner chains
+    // of several words
+    __device__ __forceinline__ double rel_dq_bf(uint64_t w) const {
+        const uint64_t u = w ^ 0xFFF0000000000000ull;
+        const bool isbin = (u & 0xFFF0000000000000ull) == 0xFFF0000000000000ull && (u & 0x000FFFFFFFFFFFFFull) != 0;
+        const uint64_t t = (u & 0x000FFFFFFFFFFFFFull) - 1u;
+        const double y = i2d_small((long long)unzz(t >> 1)) * b;
+        const double tk = y + 6755399441055744.0;
+        const double k = tk - 6755399441055744.0;
+        const double f = y - k;
+        double p = u2d(0x3D7816193166D0F9ull);
+        p = p * f; p = p + u2d(0x3DBC3BD650FC2986ull);
+        p = p * f; p = p + u2d(0x3DFE8CAC7351BB25ull);
+        p = p * f; p = p + u2d(0x3E3E4CF5158B8ECAull);
+        p = p * f; p = p + u2d(0x3E7B5253D395E7C4ull);
+        p = p * f; p = p + u2d(0x3EB62C0223A5C824ull);
+        p = p * f; p = p + u2d(0x3EEFFCBFC588B0C7ull);
+        p = p * f; p = p + u2d(0x3F2430912F86C787ull);
+        p = p * f; p = p + u2d(0x3F55D87FE78A6731ull);
+        p = p * f; p = p + u2d(0x3F83B2AB6FBA4E77ull);
+        p = p * f; p = p + u2d(0x3FAC6B08D704A0C0ull);
+        p = p * f; p = p + u2d(0x3FCEBFBDFF82C58Full);
+        p = p * f; p = p + u2d(0x3FE62E42FEFA39EFull);
+        p = p * f; p = p + 1.0;
+        long long ki = (long long)(d2u(tk) - 0x4338000000000000ull);
+        ki = ki < -1022 ? -1022 : (ki > 1023 ? 1023 : ki);       // in range: ki == k
+        double mag = p * u2d((uint64_t)(ki + 1023) << 52);
+        if (!(k <= 1023.0)) mag = u2d(0x7FF0000000000000ull);
+        else if (k < -1022.0) mag = 0.0;
+        return isbin ? u2d(d2u(mag) | (t << 63)) : u2d(u);
+    }
     __device__ __forceinline__ double rel_dq(uint64_t w) const {
         uint64_t u = w ^ 0xFFF0000000000000ull;
         if ((u & 0xFFF0000000000000ull) == 0xFFF0000000000000ull &&
