@@ -301,8 +301,9 @@ __device__ __forceinline__ void rze1_scatter(const uint32_t (&lo)[32], const uin
     for (int j = 0; j < NP; ++j) {
         const uint32_t w = j < KL ? lo[j] : hi[j - KL];
         const int b = j < KL ? j : 32 + j - KL;
+        // wor bit b is set iff some lane's plane word b is non-zero (wor is the warp's
+        // OR of the residuals)
         if (!((wor >> b) & 1u)) continue;                       // plane empty in this warp
-        if (!__any_sync(PFPL_FULL, w != 0)) continue;
         const int pl = B - 1 - b;
         const uint32_t H = nzmark(w);
         const uint32_t o = __shfl_sync(PFPL_FULL, j < KL ? offl : offh, b & 31) +
@@ -379,7 +380,6 @@ __device__ __forceinline__ void rze1_scatter_w(const uint32_t (&lo)[32], const u
             const int b = 8 * w8 + i;
             const uint32_t w = b < 32 ? lo[b & 31] : hi[b & 31];
             if (!((wor >> b) & 1u)) continue;                       // plane empty in this warp
-            if (!__any_sync(PFPL_FULL, w != 0)) continue;
             const int pl = B - 1 - b;
             const uint32_t H = nzmark(w);
             const uint32_t o = __shfl_sync(PFPL_FULL, b < 32 ? offl : offh, b & 31) +
@@ -447,7 +447,8 @@ __device__ __forceinline__ void rze1_scatter_s(uint8_t* wbuf, uint8_t* z1, uint8
     const int ng = (P + 3) >> 2;
 #pragma unroll 1
     for (int g = 0; g < ng; ++g) {
-        if (!(wor & (0xFull << (4 * g)))) continue;          // warp-uniform
+        const uint32_t wg = (uint32_t)(wor >> (4 * g)) & 0xFu;   // warp-uniform
+        if (!wg) continue;
         const uint4 v4 = *(const uint4*)plane_slot<T>(wbuf, tid, g);
         const uint32_t cnt = nzcount4(v4);
         const uint32_t ex = warp_incl_scan(cnt, lane) - cnt;
@@ -456,8 +457,7 @@ __device__ __forceinline__ void rze1_scatter_s(uint8_t* wbuf, uint8_t* z1, uint8
         for (int i = 0; i < 4; ++i) {
             const int b = 4 * g + i;
             const uint32_t w = w4[i];
-            if (!((wor >> b) & 1u)) continue;                   // plane empty in this warp
-            if (!__any_sync(PFPL_FULL, w != 0)) continue;
+            if (!((wg >> i) & 1u)) continue;                    // plane empty in this warp
             const uint32_t H = nzmark(w);
             const uint32_t o = __shfl_sync(PFPL_FULL, b < 32 ? offl : offh, b & 31) +
                                __byte_perm(ex, 0, 0x4440 + i);
