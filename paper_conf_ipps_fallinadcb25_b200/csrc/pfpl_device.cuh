@@ -380,6 +380,11 @@ template <> struct QF<float> {
     // rel_q accepts.  |L| <= 125.5 keeps pow2p away from its inf/0 clamps.  Otherwise
     // `slow` is set and the caller runs rel_q (same bits either way).
     __device__ __forceinline__ uint32_t rel_q_fast(float v, bool& slow) const {
+        bool bin;
+        return rel_q_fast(v, slow, bin);
+    }
+    // also reports whether the word is a bin (false: raw, or slow)
+    __device__ __forceinline__ uint32_t rel_q_fast(float v, bool& slow, bool& bin) const {
         // branch-free: every quantity is computed, the word is selected at the end
         const uint32_t u = f2u(v), sign = u >> 31, au = u & 0x7FFFFFFFu;
         const bool normal = au - 0x00800000u < 0x7F800000u - 0x00800000u;   // finite, not denormal/0
@@ -397,7 +402,7 @@ template <> struct QF<float> {
         // exact as a float for |k| < 2^21; the sign+exponent inversion cancels the NaN tag
         const uint32_t binw = f2u(fabsf(__fmaf_rn(k, 4.0f, 1.0f)) + 8388608.0f) - 0x4B000000u + sign;
         const uint32_t lossw = (au > 0x7F800000u ? au : u) ^ 0xFF800000u;
-        const bool bin = normal & certain & (fabsf(k) < 2097152.0f);
+        bin = normal & certain & (fabsf(k) < 2097152.0f);
         slow = normal & !certain;
         return bin ? binw : lossw;
     }
@@ -487,6 +492,10 @@ template <> struct QF<double> {
     // f64 form of QF<float>::rel_q_fast: L = exponent (exact) + lg2.approx.f32 of the
     // mantissa truncated to binary32; |L| <= 1021.5 keeps pow2p away from its clamps
     __device__ __forceinline__ uint64_t rel_q_fast(double v, bool& slow) const {
+        bool bin;
+        return rel_q_fast(v, slow, bin);
+    }
+    __device__ __forceinline__ uint64_t rel_q_fast(double v, bool& slow, bool& bin) const {
         const uint64_t u = d2u(v), sign = u >> 63, au = u & 0x7FFFFFFFFFFFFFFFull;
         const bool normal = au - 0x0010000000000000ull < 0x7FF0000000000000ull - 0x0010000000000000ull;
         const int e = (int)(au >> 52) - 1023;
@@ -502,7 +511,7 @@ template <> struct QF<double> {
         // payload 1 + (zigzag(k) << 1 | sign) = |4k + 1| + sign, exact for |k| < 2^50
         const uint64_t binw = d2u(fabs(__fma_rn(k, 4.0, 1.0)) + 4503599627370496.0) - 0x4330000000000000ull + sign;
         const uint64_t lossw = (au > 0x7FF0000000000000ull ? au : u) ^ 0xFFF0000000000000ull;
-        const bool bin = normal & certain & (fabs(k) < 1125899906842624.0);
+        bin = normal & certain & (fabs(k) < 1125899906842624.0);
         slow = normal & !certain;
         return bin ? binw : lossw;
     }

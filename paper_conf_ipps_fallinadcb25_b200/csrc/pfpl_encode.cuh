@@ -760,6 +760,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     __syncwarp();
                     uint32_t nraw = 0;
                     uint32_t slowm = 0;     // REL: values whose fast-path bin is not certain
+                    uint32_t rawm = 0;      // REL: values stored raw by the fast path
 #pragma unroll kTpUnroll
                     for (int i = 0; i < 2 * S_; ++i) {
                         const int r = sizeof(T) == 4 ? tid : 2 * tid + (i >> 3);
@@ -771,14 +772,17 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
 #pragma unroll
                         for (int k = 0; k < 16 / S_; ++k) {
                             if constexpr (MODE == MODE_REL) {
-                                bool sl;
-                                const W fw = q.rel_q_fast(x[k], sl);
+                                bool sl, bn;
+                                const W fw = q.rel_q_fast(x[k], sl, bn);
                                 // an uncertain value keeps its input bits for the exact pass
                                 W xb;
                                 memcpy(&xb, &x[k], sizeof(W));
                                 w[k] = sl ? xb : fw;
-                                slowm |= (sl ? 1u : 0u) << (i * (16 / S_) + k);
-                                nraw += (sl || is_bin_word<T, MODE>(fw, (W)qbias, raw)) ? 0u : 1u;
+                                // shift-in masks (one LEA each; value j ends at bit 31 - j):
+                                // uncertain values, and values stored raw (a non-bin word
+                                // is never in the bin range, R11)
+                                slowm = slowm * 2u + (sl ? 1u : 0u);
+                                rawm = rawm * 2u + ((sl || (bn && !raw)) ? 0u : 1u);
                             } else {
                                 w[k] = quantize_b<T, MODE>(q, x[k], raw);
                                 nraw += is_bin_word<T, MODE>(w[k], (W)qbias, raw) ? 0u : 1u;
@@ -788,6 +792,9 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         *a = v;
                     }
                     if constexpr (MODE == MODE_REL) {
+                        static_assert(2 * S_ * (16 / S_) == 32, "32 values per thread");
+                        slowm = __brev(slowm);
+                        nraw = __popc(rawm);
                         // the exact quantizer (rel_q, the format's definition) for the few
                         // uncertain values, spread over the warp's lanes: each
                         // lane lists its values (element id = 32 * lane + j) in this warp's
