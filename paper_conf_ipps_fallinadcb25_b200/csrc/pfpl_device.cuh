@@ -258,9 +258,11 @@ __device__ __forceinline__ int64_t unzz(uint64_t z) { return (int64_t)((z >> 1) 
 template <typename T> struct QF;
 template <> struct QF<float> {
     float a, b, c, m1, m2;
+    float limc;     // REL fast path: 0.5 - (m1 * 125.5 + m2) rounded down, the margin at the largest |L|
     __device__ __forceinline__ void load(const QConst& q) {
         a = u2f((uint32_t)q.a); b = u2f((uint32_t)q.b); c = u2f((uint32_t)q.c);
         m1 = u2f((uint32_t)q.m1); m2 = u2f((uint32_t)q.m2);
+        limc = __fsub_rd(0.5f, __fmaf_ru(125.5f, m1, m2));
     }
     // ABS/NOA: a = eps_eff, b = inv, c = eb2.  Bin = rint(v*inv); decode
     // immediately and keep the bin only if |v - bin*2eps| <= eps (R7);
@@ -406,6 +408,37 @@ template <> struct QF<float> {
         slow = normal & !certain;
         return bin ? binw : lossw;
     }
+    // rel_q_fast on a pair (u0, u1 the input bits): s = L*c and rint(s) on FP32x2 (the same
+    // IEEE operations as rel_q_fast); the margin is the constant limc (the bound at the
+    // largest |L|).  A slow value's word is its input bits (for the exact pass).
+    __device__ __forceinline__ uint64_t rel_q_fast2(uint32_t u0, uint32_t u1, uint64_t nz2, uint32_t& slow2,
+                                                   uint32_t& raw2) const {
+        const uint32_t au0 = u0 & 0x7FFFFFFFu, au1 = u1 & 0x7FFFFFFFu;
+        float L0, L1;
+        asm("lg2.approx.f32 %0, %1;" : "=f"(L0) : "f"(u2f(au0)));
+        asm("lg2.approx.f32 %0, %1;" : "=f"(L1) : "f"(u2f(au1)));
+        const uint64_t s = pk_mul(pk(L0, L1), pk(c, c), nz2);
+        const uint64_t ts = pk_add(s, pk(12582912.0f, 12582912.0f));
+        const uint64_t k = pk_add(ts, pk(-12582912.0f, -12582912.0f));
+        const uint64_t d = pk_sub(s, k);
+        auto one = [&](uint32_t u, uint32_t au, float L, float kf, float df, uint32_t& sl, uint32_t& rw) -> uint32_t {
+            const bool normal = au - 0x00800000u < 0x7F800000u - 0x00800000u;
+            const bool certain = (fabsf(df) <= limc) & (fabsf(L) <= 125.5f);
+            const uint32_t binw = f2u(fabsf(__fmaf_rn(kf, 4.0f, 1.0f)) + 8388608.0f) - 0x4B000000u + (u >> 31);
+            const uint32_t lossw = (au > 0x7F800000u ? au : u) ^ 0xFF800000u;
+            const bool bin = normal & certain & (fabsf(kf) < 2097152.0f);
+            const bool slw = normal & !certain;
+            sl = slw ? 1u : 0u;
+            rw = (bin | slw) ? 0u : 1u;
+            return slw ? u : (bin ? binw : lossw);
+        };
+        uint32_t sl0, sl1, rw0, rw1;
+        const uint32_t w0 = one(u0, au0, L0, pk_lo(k), pk_lo(d), sl0, rw0);
+        const uint32_t w1 = one(u1, au1, L1, pk_hi(k), pk_hi(d), sl1, rw1);
+        slow2 = sl0 | (sl1 << 1);
+        raw2 = rw0 | (rw1 << 1);
+        return ((uint64_t)w1 << 32) | w0;
+    }
     // rel_dq on a pair of words: the same IEEE operations (bin*w, rint by 1.5*2^23, f, the
     // degree-7 Horner of pow2p, the power-of-two scale), two per instruction
     __device__ __forceinline__ uint64_t rel_dq2(uint32_t w0, uint32_t w1, uint64_t nz2) const {
@@ -449,8 +482,10 @@ template <> struct QF<float> {
 };
 template <> struct QF<double> {
     double a, b, c, m1, m2;
+    double limc;    // REL fast path: 0.5 - (m1 * 1021.5 + m2) rounded down
     __device__ __forceinline__ void load(const QConst& q) {
         a = u2d(q.a); b = u2d(q.b); c = u2d(q.c); m1 = u2d(q.m1); m2 = u2d(q.m2);
+        limc = __dsub_rd(0.5, __fma_ru(1021.5, m1, m2));
     }
     __device__ __forceinline__ uint64_t abs_q(double v) const {
         double s = v * b;
@@ -505,9 +540,8 @@ template <> struct QF<double> {
         const double s = L * c;
         const double ts = s + 6755399441055744.0;
         const double k = ts - 6755399441055744.0;
-        const double aL = fabs(L);
-        const double lim = __fma_rn(-m1, aL, 0.5 - m2);
-        const bool certain = (fabs(s - k) <= lim) & (aL <= 1021.5);
+        // the margin at |L| = 1021.5 bounds every smaller |L| (m1 >= 0): one compare
+        const bool certain = (fabs(s - k) <= limc) & (fabs(L) <= 1021.5);
         // payload 1 + (zigzag(k) << 1 | sign) = |4k + 1| + sign, exact for |k| < 2^50
         const uint64_t binw = d2u(fabs(__fma_rn(k, 4.0, 1.0)) + 4503599627370496.0) - 0x4330000000000000ull + sign;
         const uint64_t lossw = (au > 0x7FF0000000000000ull ? au : u) ^ 0xFFF0000000000000ull;

@@ -87,6 +87,9 @@ __device__ __forceinline__ void q_arrive(uint32_t bar, int lane) {
         if (lane == 0) mbar_arrive(bar);
     }
 }
+#ifndef PFPL_PACKED_REL
+#define PFPL_PACKED_REL 0     // the f32 REL fast path on FP32x2 pairs (measured 5% slower: off)
+#endif
 #ifndef PFPL_PACKED_Q
 #define PFPL_PACKED_Q 1       // the f32 ABS/NOA fast-path quantizer on FFMA2/FADD2 pairs
 #endif
@@ -769,6 +772,17 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         T x[16 / S_];
                         W w[16 / S_];
                         memcpy(x, &v, 16);
+                        if constexpr (MODE == MODE_REL && sizeof(T) == 4 && PFPL_PACKED_REL) {
+                            // shift-in masks (value j ends at bit 31 - j), two values at a time
+                            uint32_t s01, r01, s23, r23;
+                            const uint64_t w01 = q.rel_q_fast2(v.x, v.y, p.nz2, s01, r01);
+                            const uint64_t w23 = q.rel_q_fast2(v.z, v.w, p.nz2, s23, r23);
+                            slowm = slowm * 16u + (__brev(s01 | (s23 << 2)) >> 28);
+                            rawm = rawm * 16u + (r01 | (r23 << 2));
+                            v = make_uint4((uint32_t)w01, (uint32_t)(w01 >> 32), (uint32_t)w23, (uint32_t)(w23 >> 32));
+                            *a = v;
+                            continue;
+                        }
 #pragma unroll
                         for (int k = 0; k < 16 / S_; ++k) {
                             if constexpr (MODE == MODE_REL) {
@@ -782,7 +796,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                                 // uncertain values, and values stored raw (a non-bin word
                                 // is never in the bin range, R11)
                                 slowm = slowm * 2u + (sl ? 1u : 0u);
-                                rawm = rawm * 2u + ((sl || (bn && !raw)) ? 0u : 1u);
+                                rawm = rawm * 2u + ((sl || bn) ? 0u : 1u);   // REL never runs in raw-words mode (host: MODE_RAW)
                             } else {
                                 w[k] = quantize_b<T, MODE>(q, x[k], raw);
                                 nraw += is_bin_word<T, MODE>(w[k], (W)qbias, raw) ? 0u : 1u;
