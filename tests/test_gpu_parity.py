@@ -374,3 +374,39 @@ def test_rel_bin_edges_and_extremes(pk, orc, dt, eps):
     cw = 16384 // np.dtype(dt).itemsize
     x = np.resize(x, ((x.size + cw - 1) // cw) * cw)     # full chunks: the fast-path layout
     _check(pk, orc, x, "rel", eps)
+
+
+def _tier_mix(dt, bound: str, eps: float, seed: int = 11) -> np.ndarray:
+    """Blocks of 1024 values (one encoder warp's share of a chunk, f32 and f64) whose
+    bin-domain residuals are ~2^k, with k cycling so that neighbouring warps of a chunk
+    sit in different transpose tiers (P <= 8, 16, 32 and, for f64, the high-half tiers)
+    and the largest k overflow into unquantizable (raw) words."""
+    rng = np.random.default_rng(seed)
+    ks = [0, 3, 5, 6, 9, 12, 14, 17, 20, 23, 26, 30] if dt == np.float32 else \
+         [0, 5, 9, 14, 20, 26, 30, 33, 36, 39, 44, 47, 52, 60]
+    order = np.concatenate([rng.permutation(len(ks)) for _ in range(8 if dt == np.float32 else 10)])
+    out = []
+    for j in order:
+        r = float(2.0 ** ks[j])
+        u = rng.uniform(-r, r, 1024) + np.arange(1024) * 0.25
+        if bound == "rel":
+            step = 2.0 * np.log2(1.0 + eps)
+            with np.errstate(over="ignore"):
+                v = np.exp2(np.clip(step * u, -2000.0, 2000.0)) * rng.choice([-1.0, 1.0], 1024)
+        else:
+            v = 2.0 * eps * u
+        out.append(v)
+    with np.errstate(over="ignore"):
+        return np.concatenate(out).astype(dt)
+
+
+@pytest.mark.parametrize("bound", ["abs", "rel", "noa"])
+@pytest.mark.parametrize("dt", [np.float32, np.float64])
+def test_every_plane_tier_per_warp(pk, orc, bound, dt):
+    """The three level-1 code shapes (one copy per tier for f32 ABS, the
+    windowed path for f32 NOA and f64 ABS/NOA, the staged path for REL) on chunks whose
+    warps run different tiers, plus a ragged tail: same bytes as the oracle."""
+    eps = 1e-2 if bound == "rel" else 1e-3
+    x = _tier_mix(dt, bound, eps)
+    _check(pk, orc, x, bound, eps)
+    _check(pk, orc, x[: x.size - 777], bound, eps)
