@@ -6,9 +6,9 @@
 //
 //   IO warp                                   compute warps (4 for f32, 2 for f64)
 //   -------                                   ------------------------------------
-//   ticket c; chunk offset from the prefix     wait for chunk k's payload; repeat
-//   sum of the stored sizes (computed   levels 4 -> 2 rebuilt top-down
-//   by size_scan_kernel just before);          with popcount prefix ranks --
+//   chunk c; its offset from the prefix sum    wait for chunk k's payload; repeat
+//   of the stored sizes (size_scan_     levels 4 -> 2 rebuilt top-down
+//   kernel, or the IO warp's own sums);        with popcount prefix ranks --
 //   validate; load the payload into a byte     every warp derives M3/M2 itself, no
 //   ring with cp.async.bulk, up to 8 chunks    barrier; zero level: gather the
 //   ahead                                      plane words from Z1, inverse shuffle in
@@ -345,16 +345,24 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
 
     if (warp == NWC) {
         // =========================== IO warp ===========================
-        // static round-robin assignment (chunk c = blockIdx.x + k * gridDim.x): the
-        // offsets are known up front (size_scan_kernel), so no ticket atomics sit on
-        // the IO warp's critical path, and the next chunk's table entries are loaded
-        // one iteration ahead
+        // static round-robin assignment (chunk c = blockIdx.x + k * gridDim.x), so no
+        // ticket atomics sit on the IO warp's critical path.
+        // d1 (the prefix sum over the stored sizes), fused: the IO warp keeps the
+        // inclusive prefix of its own previous chunk c - G and adds the G - 1 table
+        // entries in between (first chunk: the entries before it) -- independent
+        // coalesced loads of the L2-resident table, no cross-CTA dependency and no
+        // separate scan launch.  The last chunk checks the total against the payload.
         uint32_t head = 0, rel = 0;     // ring: next free byte / released up to (monotone)
         const uint64_t G = gridDim.x;
         uint64_t c = blockIdx.x;
+        // Large streams (p.offs set) take the offsets from size_scan_kernel instead, loaded
+        // one chunk ahead: there the window sums would sit on the IO warp's critical
+        // path every chunk, while the scan launch is small against the decode.
+        const bool fused = p.offs == nullptr;
+        uint64_t incl_prev = 0, from = 0;   // excl(c) = incl_prev + sum(table[from .. c))
         uint32_t size_n = 0;
         uint64_t excl_n = 0;
-        if (c < C) { size_n = p.table[c]; excl_n = p.offs[c]; }
+        if (c < C) { size_n = p.table[c]; if (!fused) excl_n = p.offs[c]; }
         for (uint32_t k = 0;; ++k, c += G) {
             const int slot = k % NQD;
             if (c >= C) {
@@ -364,14 +372,26 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
                 if (PFPL_DEC_LANE_ARRIVE || lane == 0) mbar_arrive(smem_u32(&S.full[slot]));
                 break;
             }
-            // d1: chunk offset from the size-table prefix sum (size_scan_kernel)
             const uint32_t size = size_n;
-            const uint64_t excl = excl_n;
-            if (c + G < C) { size_n = p.table[c + G]; excl_n = p.offs[c + G]; }
+            uint64_t excl = excl_n;
+            if (c + G < C) { size_n = p.table[c + G]; if (!fused) excl_n = p.offs[c + G]; }
+            if (fused) {
+                // up to 24 x 32 entries (a 740-CTA grid) in one round of independent loads
+                uint64_t part = 0;
+                for (uint64_t i0 = from + lane; i0 < c; i0 += 32 * 24) {
+#pragma unroll
+                    for (int j = 0; j < 24; ++j)
+                        if (i0 + 32 * j < c) part += p.table[i0 + 32 * j];
+                }
+                excl = incl_prev + warp_sum64(part);
+                incl_prev = excl + size;
+                from = c + 1;
+            }
             const uint32_t m = (uint32_t)min((uint64_t)CW, (uint64_t)(p.n - c * (uint64_t)CW));
             const uint32_t rawb = m * S_;
             uint32_t bad = 0;
             if (size > rawb || excl + size > p.in_bytes || (size < 4 && size != rawb)) bad = 1;
+            if (c == C - 1 && excl + size != p.in_bytes) bad = 1;    // sizes must add up to the payload
             // reserve a ring slice for the 16-byte aligned superset of the payload
             const uint8_t* g = p.in + excl;
             const uint32_t delta = (uint32_t)((uintptr_t)g & 15u);

@@ -9,6 +9,7 @@ namespace pfpl {
 
 constexpr uint32_t kChunkBytes = 16384;   // P:141 "16 kB chunks" (R19: 16384 for both dtypes)
 constexpr uint32_t kHeaderBytes = 48;     // R18
+constexpr uint64_t kFusedScanChunks = 8192;   // decoder: d1 inside the IO warps up to 128 MiB streams
 constexpr int kEPT = 32;                  // elements per thread (one 32-bit plane word)
 
 enum Mode : int { MODE_ABS = 0, MODE_REL = 1, MODE_RAW = 2, MODE_NOA = 3 };
@@ -67,7 +68,8 @@ struct DecParams {
     QConst qc;               // a/b/c as in QConst; decoder uses eb2 (ABS/NOA) or w (REL)
     int* err;                // set to PFPL_ERR_CORRUPT on malformed chunks
     uint64_t c23;            // f32 ABS: bits of 2^23 * eb2 (inf if it overflows)
-    const uint64_t* offs;    // offs[c] = byte offset of chunk c's payload (size_scan_kernel)
+    const uint64_t* offs;    // offs[c] = byte offset of chunk c's payload (size_scan_kernel), or
+                             // null: the IO warp sums the size table itself (small streams)
     unsigned int* wd;        // watchdog report (mapped host memory) or null
     // verify mode (pfpl_decompress_verify): original values and the metric accumulators
     // vm[0] max |x-y| (f64 bits), [1] max |x-y|/|x| (f64 bits), [2] sum (x-y)^2 (f64),

@@ -34,12 +34,15 @@ def _decode_status(pk, buf) -> int:
         return e.code
 
 
-def test_fuzz_large_stream_never_faults(pk):
+@pytest.mark.parametrize("rows", [128, 160])
+def test_fuzz_large_stream_never_faults(pk, rows):
     """>= 200 single-bit flips in a 128 MiB NYX-shaped stream (8192 chunks, ~11 per
     decoder CTA, so every CTA's payload ring wraps): flips aimed at the M4 bitmaps,
-    the Z4/Z3 prefixes, the size table and random payload bytes."""
+    the Z4/Z3 prefixes, the size table and random payload bytes.  128 MiB: the decoder's
+    IO warps sum the size table themselves; 160 MiB: the offsets come from
+    size_scan_kernel (pfpl_internal.h kFusedScanChunks)."""
     spec = synth.CONFIGS["nyx"]
-    x = synth.generate(spec, device="cuda", slab=(0, 128))
+    x = synth.generate(spec, device="cuda", slab=(0, rows))
     ref = pk.compress(x, "abs", 1e-3).clone()
     y0 = pk.decompress(ref).clone()
     C = x.numel() // 4096
