@@ -302,10 +302,11 @@ def test_decompress_verify_metrics(pk, orc, dt, bound):
             assert m2["violations"] == len(idx)
 
 
-def test_full_size_16gib_sampled(pk, orc):
+def test_full_size_16gib(pk, orc):
     """BASELINE.json configs[4] (16 GiB f32, n = 2^32, ABS 1E-3) at full size on one GPU, in
-    bench's launch configuration: the size table must account for the whole stream, and
-    sampled chunks (first, last, 62 random) must be byte-identical to the oracle's encoding of
+    bench's launch configuration: the size table must account for the whole stream, the whole
+    stream must equal the oracle's (when the host has ~64 GiB free) and decode to the oracle's
+    values, and sampled chunks (first, last, 62 random) must be byte-identical to the oracle's encoding of
     the same 4096 values (ABS constants depend only on eps, so a lone chunk's payload is the
     chunk's payload in any stream) and decode to the oracle's values bit for bit."""
     free, _ = torch.cuda.mem_get_info()
@@ -322,6 +323,18 @@ def test_full_size_16gib_sampled(pk, orc):
     base = 48 + 4 * C
     assert base + int(offs[-1]) == s.numel()
     y = pk.decompress(s)
+    # the whole stream against the oracle on all host cores (~25 s of CPU work), when the
+    # host has room for the field, both decodes and the stream (~50 GiB)
+    import os
+    host_free = os.sysconf("SC_AVPHYS_PAGES") * os.sysconf("SC_PAGE_SIZE")
+    if host_free >= 64 * 2**30:
+        nt = max(1, len(os.sched_getaffinity(0)))
+        xh = x.cpu().numpy()
+        s_orc = orc.compress(xh, "abs", 1e-3, nthreads=nt)
+        assert s.cpu().numpy().tobytes() == s_orc          # all 1,048,576 chunks
+        y_orc = orc.decompress(s_orc, nthreads=nt)
+        assert np.array_equal(y.cpu().numpy().view(np.uint32), y_orc.view(np.uint32))
+        del xh, s_orc, y_orc
     rng = np.random.default_rng(4)
     for c in [0, C - 1] + list(rng.integers(1, C - 1, size=62)):
         c = int(c)
