@@ -259,10 +259,12 @@ template <typename T> struct QF;
 template <> struct QF<float> {
     float a, b, c, m1, m2;
     float limc;     // REL fast path: 0.5 - (m1 * 125.5 + m2) rounded down, the margin at the largest |L|
+    float lmax;     // REL fast path: largest certified |L|: 125.5, and |L| * c <= 2^20 so |k| < 2^21
     __device__ __forceinline__ void load(const QConst& q) {
         a = u2f((uint32_t)q.a); b = u2f((uint32_t)q.b); c = u2f((uint32_t)q.c);
         m1 = u2f((uint32_t)q.m1); m2 = u2f((uint32_t)q.m2);
         limc = __fsub_rd(0.5f, __fmaf_ru(125.5f, m1, m2));
+        lmax = fminf(125.5f, __fdiv_rd(1048576.0f, c));
     }
     // ABS/NOA: a = eps_eff, b = inv, c = eb2.  Bin = rint(v*inv); decode
     // immediately and keep the bin only if |v - bin*2eps| <= eps (R7);
@@ -408,6 +410,29 @@ template <> struct QF<float> {
         slow = normal & !certain;
         return bin ? binw : lossw;
     }
+    // rel_q_fast in the form the encoder's REL loop uses: the word of a certain bin, the
+    // lossless word of a zero / denormal / inf / NaN, and the input bits of an uncertain
+    // (slow) value, which sets `slow`; `nraw` counts the lossless ones.  |L| <= lmax also keeps |k| < 2^21, so one compare replaces rel_q_fast's |k|
+    // test (the margin stays m1 |L| + m2: the constant bound at |L| = 125.5 sends ~18% of
+    // the values of a 1E-3 field to the exact pass).  lg2.approx.ftz: L of a zero / denormal is -inf, of inf +inf,
+    // of NaN NaN, so `certain` implies a normal input.
+    __device__ __forceinline__ uint32_t rel_q_fast_w(float v, bool& slow, uint32_t& nraw) const {
+        const uint32_t u = f2u(v), au = u & 0x7FFFFFFFu;
+        const bool normal = au - 0x00800000u < 0x7F800000u - 0x00800000u;
+        float L;
+        asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(L) : "f"(u2f(au)));
+        const float s = L * c;
+        const float ts = s + 12582912.0f;
+        const float k = ts - 12582912.0f;
+        const float aL = fabsf(L);
+        const float lim = __fmaf_rn(-m1, aL, 0.5f - m2);      // margin arithmetic only
+        const bool certain = (fabsf(s - k) <= lim) & (aL <= lmax);
+        const uint32_t binw = f2u(fabsf(__fmaf_rn(k, 4.0f, 1.0f)) + 8388608.0f) - 0x4B000000u + (u >> 31);
+        const uint32_t lossw = (au > 0x7F800000u ? au : u) ^ 0xFF800000u;
+        slow = normal & !certain;
+        nraw += normal ? 0u : 1u;
+        return certain ? binw : (normal ? u : lossw);
+    }
     // rel_q_fast on a pair (u0, u1 the input bits): s = L*c and rint(s) on FP32x2 (the same
     // IEEE operations as rel_q_fast); the margin is the constant limc (the bound at the
     // largest |L|).  A slow value's word is its input bits (for the exact pass).
@@ -483,9 +508,11 @@ template <> struct QF<float> {
 template <> struct QF<double> {
     double a, b, c, m1, m2;
     double limc;    // REL fast path: 0.5 - (m1 * 1021.5 + m2) rounded down
+    double lmax;    // REL fast path: largest certified |L|: 1021.5, and |L| * c <= 2^49 so |k| < 2^50
     __device__ __forceinline__ void load(const QConst& q) {
         a = u2d(q.a); b = u2d(q.b); c = u2d(q.c); m1 = u2d(q.m1); m2 = u2d(q.m2);
         limc = __dsub_rd(0.5, __fma_ru(1021.5, m1, m2));
+        lmax = fmin(1021.5, __ddiv_rd(562949953421312.0, c));
     }
     __device__ __forceinline__ uint64_t abs_q(double v) const {
         double s = v * b;
@@ -548,6 +575,25 @@ template <> struct QF<double> {
         bin = normal & certain & (fabs(k) < 1125899906842624.0);
         slow = normal & !certain;
         return bin ? binw : lossw;
+    }
+    // f64 form of QF<float>::rel_q_fast_w (L of a zero / denormal has |L| >= 1022, of an
+    // inf / NaN >= 1024, so `certain` implies a normal input)
+    __device__ __forceinline__ uint64_t rel_q_fast_w(double v, bool& slow, uint32_t& nraw) const {
+        const uint64_t u = d2u(v), au = u & 0x7FFFFFFFFFFFFFFFull;
+        const bool normal = au - 0x0010000000000000ull < 0x7FF0000000000000ull - 0x0010000000000000ull;
+        const int e = (int)(au >> 52) - 1023;
+        float lm;
+        asm("lg2.approx.f32 %0, %1;" : "=f"(lm) : "f"(u2f(0x3F800000u | (uint32_t)((au >> 29) & 0x7FFFFFu))));
+        const double L = i2d_small(e) + (double)lm;
+        const double s = L * c;
+        const double ts = s + 6755399441055744.0;
+        const double k = ts - 6755399441055744.0;
+        const bool certain = (fabs(s - k) <= limc) & (fabs(L) <= lmax);
+        const uint64_t binw = d2u(fabs(__fma_rn(k, 4.0, 1.0)) + 4503599627370496.0) - 0x4330000000000000ull + (u >> 63);
+        const uint64_t lossw = (au > 0x7FF0000000000000ull ? au : u) ^ 0xFFF0000000000000ull;
+        slow = normal & !certain;
+        nraw += normal ? 0u : 1u;
+        return certain ? binw : (normal ? u : lossw);
     }
     // rel_dq without branches (the same IEEE operations; non-bin words compute a
     // discarded value), so the decoder can interleave the 26-operation Horner chains

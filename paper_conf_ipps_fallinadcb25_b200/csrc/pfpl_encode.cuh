@@ -90,6 +90,9 @@ __device__ __forceinline__ void q_arrive(uint32_t bar, int lane) {
 #ifndef PFPL_PACKED_REL
 #define PFPL_PACKED_REL 0     // the f32 REL fast path on FP32x2 pairs (measured 5% slower: off)
 #endif
+#ifndef PFPL_REL_FASTW
+#define PFPL_REL_FASTW 1       // REL fast path: rel_q_fast_w (ftz lg2, one |L| compare, lossless values counted)
+#endif
 #ifndef PFPL_PACKED_Q
 #define PFPL_PACKED_Q 1       // the f32 ABS/NOA fast-path quantizer on FFMA2/FADD2 pairs
 #endif
@@ -785,7 +788,11 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         }
 #pragma unroll
                         for (int k = 0; k < 16 / S_; ++k) {
-                            if constexpr (MODE == MODE_REL) {
+                            if constexpr (MODE == MODE_REL && PFPL_REL_FASTW) {
+                                bool sl;
+                                w[k] = q.rel_q_fast_w(x[k], sl, nraw);
+                                slowm = slowm * 2u + (sl ? 1u : 0u);     // shift-in mask (one LEA)
+                            } else if constexpr (MODE == MODE_REL) {
                                 bool sl, bn;
                                 const W fw = q.rel_q_fast(x[k], sl, bn);
                                 // an uncertain value keeps its input bits for the exact pass
@@ -808,7 +815,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                     if constexpr (MODE == MODE_REL) {
                         static_assert(2 * S_ * (16 / S_) == 32, "32 values per thread");
                         slowm = __brev(slowm);
-                        nraw = __popc(rawm);
+                        if (!PFPL_REL_FASTW) nraw = __popc(rawm);
                         // the exact quantizer (rel_q, the format's definition) for the few
                         // uncertain values, spread over the warp's lanes: each
                         // lane lists its values (element id = 32 * lane + j) in this warp's
