@@ -613,7 +613,26 @@ def _identity_check(pk, synth, pdist, dist, spec, args, r, out, nch, rank, world
             toff += 4 * nq
             poff += r.sizes[q]
         ok = ok and all(per_rank) and poff == single.numel()
+        # the same workload on this one GPU (context for the driver's scaling numbers, which
+        # compare against the N = 1 line; that line is the NYX headline workload)
+        outb = torch.empty(pk.max_compressed_bytes(full.numel(), full.dtype), dtype=torch.uint8, device=dev)
+        rcv = torch.zeros(4, dtype=torch.int64, device=dev)
+        ts = []
+        for i in range(4):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            pk.compress_async(full, outb, rcv, args.bound, args.eps, stream=stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            if i:
+                ts.append(e0.elapsed_time(e1))
+        one_gpu = {"compress_gbs": spec.n * spec.itemsize / (statistics.median(ts) * 1e-3) / 1e9,
+                   "what": "rank 0 alone, one GPU, the whole field of this line's workload, "
+                           "pfpl_compress_async between CUDA events, median of 3 after 1 warm-up "
+                           "(the N = 1 bench line is the NYX headline workload instead)"}
+        del outb, rcv
         res = {"identical_to_single_gpu_stream": bool(ok), "per_rank": per_rank,
+               "single_gpu_same_workload": one_gpu,
                "stream_bytes": int(single.numel()),
                "method": "rank 0: pfpl_compress of the whole field on one GPU; header, total size and "
                          "64-bit checksums of every rank's table slice and payload vs the same byte "
