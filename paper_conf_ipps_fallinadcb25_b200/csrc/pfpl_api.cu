@@ -51,6 +51,21 @@ unsigned int* g_wd_host = nullptr;     // mapped pinned watchdog report {site, b
 unsigned int* g_wd_dev = nullptr;
 
 std::once_flag g_wd_once;
+// f32 ABS encoder form hint (pfpl_encode.cuh, encode_kernel): one mapped host word per
+// process, written by CTA 0 of every f32 ABS launch, read here without a sync (so a hint
+// takes effect from the next call; both forms write the same bytes)
+std::once_flag g_x0_once;
+unsigned int* g_x0_host = nullptr;
+unsigned int* g_x0_dev = nullptr;
+unsigned int* x0_hint_ptr() {
+    std::call_once(g_x0_once, [] {
+        if (cudaHostAlloc(&g_x0_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_x0_host = nullptr; return; }
+        memset(g_x0_host, 0, 64);
+        if (cudaHostGetDevicePointer(&g_x0_dev, g_x0_host, 0) != cudaSuccess) g_x0_dev = nullptr;
+    });
+    return g_x0_dev;
+}
+
 unsigned int* watchdog_ptr() {
     std::call_once(g_wd_once, [] {
         if (cudaHostAlloc(&g_wd_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_wd_host = nullptr; return; }
@@ -273,9 +288,14 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
     p.stats = st_cur;
     p.stats_next = st_next;
     p.nz2 = 0x8000000080000000ull;
+    bool x0 = false;
+    if (dtype == PFPL_F32 && mode == MODE_ABS) {
+        p.x0_hint = x0_hint_ptr();
+        x0 = p.x0_hint && *(volatile unsigned int*)g_x0_host == 1u;
+    }
     const bool ms = (opts & PFPL_OPT_MS_RESIDUALS) != 0;
     const int grid = encode_grid(dtype, mode, ms, C);
-    CK(launch_encode(dtype, mode, ms, p, grid, s));
+    CK(launch_encode(dtype, mode, ms, x0, p, grid, s));
     g_launches += 1;
     // each persistent encoder CTA consumes (stages + 1) tickets per pipeline beyond its chunks
     sc->ticket_val += C + (uint64_t)grid * (uint64_t)encode_tickets_per_cta(dtype);
@@ -751,6 +771,9 @@ int pfpl_last_stats(void* stream, uint64_t* unquantizable, uint64_t* raw_chunks)
 }
 
 uint64_t pfpl_launch_count(void) { return g_launches.load(); }
+int pfpl_f32_abs_form(void) {
+    return g_x0_host && *(volatile unsigned int*)g_x0_host == 1u ? 1 : 0;
+}
 
 const char* pfpl_version(void) { return "pfpl-b200 1.0 sm_100a (stream format v1)"; }
 

@@ -93,6 +93,9 @@ __device__ __forceinline__ void q_arrive(uint32_t bar, int lane) {
 #ifndef PFPL_REL_FASTW
 #define PFPL_REL_FASTW 1       // REL fast path: rel_q_fast_w (ftz lg2, one |L| compare, lossless values counted)
 #endif
+#ifndef PFPL_X0
+#define PFPL_X0 1             // f32 ABS: a second encoder form with the first-residual split
+#endif
 #ifndef PFPL_PACKED_Q
 #define PFPL_PACKED_Q 1       // the f32 ABS/NOA fast-path quantizer on FFMA2/FADD2 pairs
 #endif
@@ -113,6 +116,7 @@ struct EncShared {
     uint8_t wcnt[128];               // per-warp per-plane Z1 counts, [warp * B + bit]
     uint32_t scan2[4];               // level-2 warp totals
     uint32_t head, rel;                // arena: next free byte / released up to (monotone counters)
+    uint32_t xh;                       // X0 form: extra planes of the chunk's first residual
     unsigned long long in_c[NIN];
     QEntry q[NQ];
     unsigned long long full[NIN], mq_full[NQ], mq_empty[NQ];
@@ -547,7 +551,28 @@ __device__ __forceinline__ bool is_bin_word(typename Tr<T>::W w, typename Tr<T>:
 }
 
 // [stage] kernel setup + tickets
-template <typename T, int MODE, bool MSR>
+// the hint for the next f32 ABS call (IO warp of CTA 0, off the compute warps' code): the
+// split form pays when chunks start with a large bin on a smooth field, i.e. first residuals
+// reach 2^8 while the others stay below: at >= 4 of 8 chunk starts |bin| = |v| / (2 eps) >= 64
+// and the next value is within 4 bins of it (on a rough field the other residuals keep warp 0
+// wide anyway, and there the plain form is faster: the rough NYX variant's neighbours are
+// 3-70 bins apart)
+__device__ __forceinline__ void x0_hint_update(const EncParams& p) {
+    const float b = u2f((uint32_t)p.qc.b);
+    int big = 0;
+    for (int k = 0; k < 8; ++k) {
+        const uint64_t e = (p.C * (uint64_t)k / 8u) * 4096u;
+        if (e + 1 >= p.n) continue;
+        const float v0 = ((const float*)p.in)[e], v1 = ((const float*)p.in)[e + 1];
+        big += (fabsf(v0) * b >= 64.0f && fabsf(v1 - v0) * b < 4.0f) ? 1 : 0;    // NaN: no
+    }
+    *(volatile unsigned int*)p.x0_hint = big >= 4 ? 1u : 0u;
+}
+
+// X0 selects the form with the first-residual split (kX0 below); both forms write the same
+// bytes.  The host picks the form from a hint that CTA 0 of every f32 ABS launch leaves in
+// mapped host memory (x0_hint_of below), so a hint takes effect from the next call.
+template <typename T, int MODE, bool MSR, bool X0>
 __global__ void __launch_bounds__(Tr<T>::NT + 32, EncCfg<T>::MINB)
 encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
@@ -601,6 +626,8 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     if (warp == NWC) {
 // [stage] IO warp: queue
         // =========================== IO warp ===========================
+        if (sizeof(T) == 4 && MODE == MODE_ABS && PFPL_X0 && p.x0_hint && blockIdx.x == 0 && lane == 0)
+            x0_hint_update(p);
         const uint64_t EP = (uint64_t)p.epoch << 48;
         for (uint32_t k = 0;; ++k) {
             const int slot = k % NQ;
@@ -675,6 +702,15 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     // bias of quantize_b(): only the f32 ABS/NOA bin path is biased
     const uint64_t qbias = (sizeof(T) == 4 && (MODE == MODE_ABS || (MODE == MODE_NOA && !raw)))
                                ? 0x4B000000ull : 0ull;
+    // kX0 (f32 ABS fast path, the X0 form): the chunk's first residual x0 is taken against
+    // q[-1] = 0, so it carries the whole first bin and alone would lift warp 0 out of
+    // the 8-plane tier.  When every other residual of warp 0 is below 2^8, its bits >= 8
+    // become "extra" planes, in which only element 0 is set: one byte 0x01 at the start of
+    // warp 0's segment of the plane (R13) and M1 byte 0x01, added outside the tiered level-1
+    // code (counts when the offsets are formed, bytes right after).  The decision is a vote
+    // taken before the warp OR is reduced.  Same bytes as the plain shuffle.
+    constexpr bool kX0 = X0 && sizeof(T) == 4 && MODE == MODE_ABS &&
+                         !(PFPL_UNIFIED_L1 == 1) && !PFPL_TIER4 && PFPL_MIN_TIER <= 8;
     uint32_t it = 0;
     for (;; ++it) {
         const int s = it % NIN;
@@ -701,6 +737,9 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             const uint32_t t = __reduce_add_sync(PFPL_FULL, nraw);
             if (lane == 0 && t && p.stats) atomicAdd(&p.stats[0], (unsigned long long)t);
         };
+        // kX0: warp 0's extra planes of this chunk, read by every warp after the counts barrier
+        // (0 unless the fast path splits x0)
+        if (kX0 && tid == 0) S.xh = 0u;
         {
             // biased words (quantize_b): q + bias; the bias cancels in q[i] - q[i-1]
             W qprev = (W)qbias;
@@ -732,12 +771,22 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
                         const uint32_t r0 = rcode<MSR>(z0 - zp), r1 = rcode<MSR>(z1 - z0);
                         const uint32_t r2 = rcode<MSR>(z2 - z1), r3 = rcode<MSR>(z3 - z2);
                         zp = z3;
-                        orw |= r0 | r1;
+                        orw |= (kX0 && i == 0 ? 0u : r0) | r1;    // kX0: lo[0] is ORed after the loop
                         orw |= r2 | r3;
                         lo[4 * i] = r0; lo[4 * i + 1] = r1; lo[4 * i + 2] = r2; lo[4 * i + 3] = r3;
                     }
                     done = __all_sync(PFPL_FULL, ok[0] && ok[1] && ok[2] && ok[3] && ok[4] && ok[5] &&
                                                      ok[6] && ok[7]);
+                    if constexpr (kX0) {
+                        // every residual of the warp below 2^8, x0's bits >= 8 aside?
+                        const bool small = __all_sync(PFPL_FULL, (orw | (tid ? lo[0] : lo[0] & 0xFFu)) < 256u);
+                        if (tid == 0) {
+                            const uint32_t xh = (done && small) ? lo[0] & ~0xFFu : 0u;
+                            lo[0] ^= xh;
+                            S.xh = xh;
+                        }
+                        orw |= lo[0];          // x0 whole unless split (a failed fast path redoes lo[])
+                    }
                     orv = (W)orw;
                 }
             }
@@ -984,11 +1033,12 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
         // Z1 offsets of this warp's segments: planes in decreasing bit order,
         // then warps (lane l owns bit l and 32+l)
         uint32_t offl, offh, n1, head;
+        const uint32_t xsw = kX0 ? S.xh : 0u;     // kX0: warp 0's extra planes (every warp reads it)
         {
             uint32_t myl = 0, myh = 0, tl = 0, th = 0;
 #pragma unroll
             for (int w = 0; w < NWC; ++w) {
-                const uint32_t a = S.wcnt[w * B + lane];
+                const uint32_t a = S.wcnt[w * B + lane] + ((kX0 && w == 0) ? (xsw >> lane) & 1u : 0u);
                 const uint32_t b = B == 64 ? S.wcnt[w * B + 32 + lane] : 0u;
                 if (w < warp) { myl += a; myh += b; }
                 tl += a;
@@ -1009,6 +1059,12 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
             head = slice_start<ARENA>(S, n1, it);
         }
         uint8_t* const z1 = arena + head % ARENA;
+        if (kX0 && warp == 0 && ((xsw >> lane) & 1u)) {
+            // extra plane `lane`: byte 0x01 at the start of warp 0's segment (offl of this
+            // lane) and M1 byte 0x01
+            z1[offl] = 1;
+            m1[(B - 1 - lane) * (CW / 64)] = 1;
+        }
 // [stage] level 1: Z1/M1 scatter
         if constexpr (kStg) {
             rze1_scatter_s<T>(sbuf, z1, m1, tid, lane, wor, P, offl, offh);

@@ -9,15 +9,15 @@ namespace pfpl {
 // host side
 // ---------------------------------------------------------------------------
 // one instantiation TU per (dtype, mode): pfpl_enc_inst.cu built with -DPFPL_DT/-DPFPL_MODE
-#define PFPL_DECL(D, M) void* enc_ptr_##D##_##M(bool ms);
+#define PFPL_DECL(D, M) void* enc_ptr_##D##_##M(bool ms, bool x0);
 PFPL_DECL(0, 0) PFPL_DECL(0, 1) PFPL_DECL(0, 2) PFPL_DECL(0, 3)
 PFPL_DECL(1, 0) PFPL_DECL(1, 1) PFPL_DECL(1, 2) PFPL_DECL(1, 3)
 #undef PFPL_DECL
 
-static void* pick_enc(int dtype, int mode, bool ms) {
-    static void* (*const tab[2][4])(bool) = {{enc_ptr_0_0, enc_ptr_0_1, enc_ptr_0_2, enc_ptr_0_3},
+static void* pick_enc(int dtype, int mode, bool ms, bool x0 = false) {
+    static void* (*const tab[2][4])(bool, bool) = {{enc_ptr_0_0, enc_ptr_0_1, enc_ptr_0_2, enc_ptr_0_3},
                                             {enc_ptr_1_0, enc_ptr_1_1, enc_ptr_1_2, enc_ptr_1_3}};
-    return tab[dtype ? 1 : 0][mode & 3](ms);
+    return tab[dtype ? 1 : 0][mode & 3](ms, x0);
 }
 
 static int enc_threads(int dtype) { return dtype == 0 ? EncCfg<float>::THREADS : EncCfg<double>::THREADS; }
@@ -80,17 +80,17 @@ cudaError_t make_row_tmap(const void* base, uint64_t bytes, CUtensorMap* map) {
     return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
-cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int grid,
+cudaError_t launch_encode(int dtype, int mode, bool ms, bool x0, const EncParams& p, int grid,
                           cudaStream_t s) {
     alignas(64) CUtensorMap map;
     cudaError_t e = make_row_tmap(p.in, p.n * (dtype == 0 ? 4u : 8u), &map);
     if (e != cudaSuccess) return e;
-    void* fn = pick_enc(dtype, mode, ms);
-    static bool prepared[2][4][2] = {};
-    if (!prepared[dtype][mode][ms]) {
+    void* fn = pick_enc(dtype, mode, ms, x0);
+    static bool prepared[2][4][2][2] = {};
+    if (!prepared[dtype][mode][ms][x0]) {
         e = prepare_enc(fn, dtype);
         if (e != cudaSuccess) return e;
-        prepared[dtype][mode][ms] = true;
+        prepared[dtype][mode][ms][x0] = true;
     }
     void* args[] = {(void*)&p, (void*)&map};
     return cudaLaunchKernel(fn, dim3(grid), dim3(enc_threads(dtype)), args, enc_smem(dtype), s);

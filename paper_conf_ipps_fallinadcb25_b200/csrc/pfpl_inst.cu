@@ -21,8 +21,14 @@ typedef float InstT;
 typedef double InstT;
 #endif
 #if PFPL_KIND == 0
-void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms) {
-    return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false>;
+// encoder: (residual code, first-residual split form; the latter exists for f32 ABS only)
+void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms, bool x0) {
+#if PFPL_DT == 0 && PFPL_MODE == 0
+    if (x0) return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, true> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, true>;
+#else
+    (void)x0;
+#endif
+    return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, false> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, false>;
 }
 #else
 // decoder: (residual code, verify mode); verify is instantiated for the default residuals

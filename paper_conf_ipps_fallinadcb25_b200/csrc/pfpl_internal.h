@@ -52,6 +52,7 @@ struct EncParams {
     unsigned long long* stats;       // [0] unquantizable values, [1] raw chunks (this call)
     unsigned long long* stats_next;  // the other slot: zeroed for the next call
     uint64_t nz2;            // two binary32 -0.0 (0x8000000080000000), opaque to ptxas: see pk_mul
+    unsigned int* x0_hint;   // f32 ABS: mapped host word, 1 = the next call should use the split form
 };
 
 struct DecParams {
@@ -82,7 +83,7 @@ struct DecParams {
 };
 
 // kernel launchers (pfpl_kernels.cu)
-cudaError_t launch_encode(int dtype, int mode, bool ms, const EncParams& p, int grid,
+cudaError_t launch_encode(int dtype, int mode, bool ms, bool x0, const EncParams& p, int grid,
                           cudaStream_t s);
 cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
                           cudaStream_t s);   // p.orig != null selects the verify kernel

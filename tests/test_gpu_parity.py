@@ -423,3 +423,21 @@ def test_every_plane_tier_per_warp(pk, orc, bound, dt):
     x = _tier_mix(dt, bound, eps)
     _check(pk, orc, x, bound, eps)
     _check(pk, orc, x[: x.size - 777], bound, eps)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("ms", [False, True])
+def test_f32_abs_both_encoder_forms(pk, orc, ms):
+    """The f32 ABS encoder's two forms (the first residual of a chunk, taken
+    against q[-1] = 0, split into single-byte extra planes, or not) write the
+    oracle's bytes.  A large-magnitude smooth field leaves the hint for the split form, a
+    small-magnitude one for the plain form, so this sequence runs both."""
+    n = 4096 * 300 + 77
+    xb = synth.generate(synth.FieldSpec("t", (n,), "f32", 11, A=0.4, tau=0.001)).numpy()
+    xs = synth.generate(synth.FieldSpec("t", (n,), "f32", 12, A=0.02, tau=0.001)).numpy()
+    forms = []
+    for x in (xb, xb, xs, xs, xb, xb):
+        forms.append(pk.f32_abs_form())
+        _check(pk, orc, x, "abs", 1e-3, ms=ms)
+    assert forms[1] == 1 and forms[3] == 0 and forms[5] == 1, forms
+
