@@ -229,13 +229,14 @@ int pfpl_last_stats(void* stream, uint64_t* unquantizable, uint64_t* raw_chunks)
 /* Number of kernel launches issued by the library since load (for bench's
  * gpu_launches claim). */
 uint64_t pfpl_launch_count(void);
-/* The form the next f32 ABS compression will run (both write the same bytes):
- * 1 = the encoder that stores a chunk's first residual (taken against q[-1] = 0) in
- * single-byte extra planes instead of widening warp 0's bit-plane tier, 0 = the plain
- * encoder.  Every f32 ABS launch leaves this hint for the next one from 8 samples of its
- * input (large first bins on a smooth field -> 1).  Host-only read of mapped memory; no
- * sync, no error. */
-int pfpl_f32_abs_form(void);
+/* The form the next f32 compression with bound `bound` (PFPL_ABS or PFPL_NOA) will run
+ * (both forms write the same bytes): 1 = the encoder that stores a chunk's first
+ * residual (taken against q[-1] = 0) in single-byte extra planes instead of widening
+ * warp 0's bit-plane tier, 0 = the plain encoder.  Every f32 ABS / NOA launch leaves this
+ * hint for the next one of its bound from 8 samples of its input (large first bins on a
+ * smooth field -> 1).  Host-only read of mapped memory; no sync.  Returns 0 for any other
+ * bound. */
+int pfpl_f32_encoder_form(int bound);
 /* Build identification string ("pfpl-b200 sm_100a ..."). */
 const char* pfpl_version(void);
 

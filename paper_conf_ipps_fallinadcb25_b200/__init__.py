@@ -70,7 +70,7 @@ def lib():
             "pfpl_watchdog_report": (i32, [ctypes.POINTER(ctypes.c_uint)]),
             "pfpl_release_scratch": (i32, []),
             "pfpl_launch_count": (u64, []),
-            "pfpl_f32_abs_form": (ctypes.c_int, []),
+            "pfpl_f32_encoder_form": (ctypes.c_int, [ctypes.c_int]),
             "pfpl_last_stats": (i32, [vp, pu64, pu64]),
             "pfpl_decompress_verify": (i32, [vp, u64, vp, vp, pu64, vp, vp]),
             "pfpl_version": (ctypes.c_char_p, []),
@@ -380,6 +380,7 @@ def launch_count() -> int:
     return int(lib().pfpl_launch_count())
 
 
-def f32_abs_form() -> int:
-    """1 if the next f32 ABS compression runs the first-residual split encoder (same bytes)."""
-    return int(lib().pfpl_f32_abs_form())
+def f32_encoder_form(bound="abs") -> int:
+    """1 if the next f32 compression with this bound (abs / noa) runs the first-residual
+    split encoder (same bytes)."""
+    return int(lib().pfpl_f32_encoder_form(_bound(bound)))

@@ -289,9 +289,12 @@ int enqueue_compress(const void* in, uint64_t n, uint64_t n_total, int dtype, in
     p.stats_next = st_next;
     p.nz2 = 0x8000000080000000ull;
     bool x0 = false;
-    if (dtype == PFPL_F32 && mode == MODE_ABS) {
-        p.x0_hint = x0_hint_ptr();
-        x0 = p.x0_hint && *(volatile unsigned int*)g_x0_host == 1u;
+    if (dtype == PFPL_F32 && (mode == MODE_ABS || mode == MODE_NOA)) {
+        // one hint word per bound (ABS, NOA): their bins differ on the same field
+        const int k = mode == MODE_NOA ? 1 : 0;
+        unsigned int* const h = x0_hint_ptr();
+        p.x0_hint = h ? h + k : nullptr;
+        x0 = p.x0_hint && ((volatile unsigned int*)g_x0_host)[k] == 1u;
     }
     const bool ms = (opts & PFPL_OPT_MS_RESIDUALS) != 0;
     const int grid = encode_grid(dtype, mode, ms, C);
@@ -771,8 +774,9 @@ int pfpl_last_stats(void* stream, uint64_t* unquantizable, uint64_t* raw_chunks)
 }
 
 uint64_t pfpl_launch_count(void) { return g_launches.load(); }
-int pfpl_f32_abs_form(void) {
-    return g_x0_host && *(volatile unsigned int*)g_x0_host == 1u ? 1 : 0;
+int pfpl_f32_encoder_form(int bound) {
+    if (!g_x0_host || (bound != PFPL_ABS && bound != PFPL_NOA)) return 0;
+    return ((volatile unsigned int*)g_x0_host)[bound == PFPL_NOA ? 1 : 0] == 1u ? 1 : 0;
 }
 
 const char* pfpl_version(void) { return "pfpl-b200 1.0 sm_100a (stream format v1)"; }

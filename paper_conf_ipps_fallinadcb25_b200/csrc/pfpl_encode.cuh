@@ -557,8 +557,7 @@ __device__ __forceinline__ bool is_bin_word(typename Tr<T>::W w, typename Tr<T>:
 // and the next value is within 4 bins of it (on a rough field the other residuals keep warp 0
 // wide anyway, and there the plain form is faster: the rough NYX variant's neighbours are
 // 3-70 bins apart)
-__device__ __forceinline__ void x0_hint_update(const EncParams& p) {
-    const float b = u2f((uint32_t)p.qc.b);
+__device__ __forceinline__ void x0_hint_update(const EncParams& p, float b) {
     int big = 0;
     for (int k = 0; k < 8; ++k) {
         const uint64_t e = (p.C * (uint64_t)k / 8u) * 4096u;
@@ -626,8 +625,9 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     if (warp == NWC) {
 // [stage] IO warp: queue
         // =========================== IO warp ===========================
-        if (sizeof(T) == 4 && MODE == MODE_ABS && PFPL_X0 && p.x0_hint && blockIdx.x == 0 && lane == 0)
-            x0_hint_update(p);
+        if (sizeof(T) == 4 && (MODE == MODE_ABS || MODE == MODE_NOA) && PFPL_X0 && p.x0_hint &&
+            blockIdx.x == 0 && lane == 0)
+            x0_hint_update(p, u2f((uint32_t)qc.b));     // NOA: the device-derived constants
         const uint64_t EP = (uint64_t)p.epoch << 48;
         for (uint32_t k = 0;; ++k) {
             const int slot = k % NQ;
@@ -709,7 +709,7 @@ encode_kernel(const EncParams p, const __grid_constant__ CUtensorMap tmap) {
     // warp 0's segment of the plane (R13) and M1 byte 0x01, added outside the tiered level-1
     // code (counts when the offsets are formed, bytes right after).  The decision is a vote
     // taken before the warp OR is reduced.  Same bytes as the plain shuffle.
-    constexpr bool kX0 = X0 && sizeof(T) == 4 && MODE == MODE_ABS &&
+    constexpr bool kX0 = X0 && sizeof(T) == 4 && (MODE == MODE_ABS || MODE == MODE_NOA) &&
                          !(PFPL_UNIFIED_L1 == 1) && !PFPL_TIER4 && PFPL_MIN_TIER <= 8;
     uint32_t it = 0;
     for (;; ++it) {

@@ -23,7 +23,7 @@ typedef double InstT;
 #if PFPL_KIND == 0
 // encoder: (residual code, first-residual split form; the latter exists for f32 ABS only)
 void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms, bool x0) {
-#if PFPL_DT == 0 && PFPL_MODE == 0
+#if PFPL_DT == 0 && (PFPL_MODE == 0 || PFPL_MODE == 3)
     if (x0) return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, true> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, true>;
 #else
     (void)x0;

@@ -426,8 +426,9 @@ def test_every_plane_tier_per_warp(pk, orc, bound, dt):
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("bound", ["abs", "noa"])
 @pytest.mark.parametrize("ms", [False, True])
-def test_f32_abs_both_encoder_forms(pk, orc, ms):
+def test_f32_abs_both_encoder_forms(pk, orc, ms, bound):
     """The f32 ABS encoder's two forms (the first residual of a chunk, taken
     against q[-1] = 0, split into single-byte extra planes, or not) write the
     oracle's bytes.  A large-magnitude smooth field leaves the hint for the split form, a
@@ -435,9 +436,14 @@ def test_f32_abs_both_encoder_forms(pk, orc, ms):
     n = 4096 * 300 + 77
     xb = synth.generate(synth.FieldSpec("t", (n,), "f32", 11, A=0.4, tau=0.001)).numpy()
     xs = synth.generate(synth.FieldSpec("t", (n,), "f32", 12, A=0.02, tau=0.001)).numpy()
+    if bound == "noa":
+        # NOA bins are relative to the range: a large relative bound keeps them small
+        eb, es = 1e-4, 1e-1
+    else:
+        eb, es = 1e-3, 1e-3
     forms = []
-    for x in (xb, xb, xs, xs, xb, xb):
-        forms.append(pk.f32_abs_form())
-        _check(pk, orc, x, "abs", 1e-3, ms=ms)
+    for x, e in ((xb, eb), (xb, eb), (xs, es), (xs, es), (xb, eb), (xb, eb)):
+        forms.append(pk.f32_encoder_form(bound))
+        _check(pk, orc, x, bound, e, ms=ms)
     assert forms[1] == 1 and forms[3] == 0 and forms[5] == 1, forms
 
