@@ -59,7 +59,7 @@ unsigned int* g_x0_host = nullptr;
 unsigned int* g_x0_dev = nullptr;
 unsigned int* x0_hint_ptr() {
     std::call_once(g_x0_once, [] {
-        if (cudaHostAlloc(&g_x0_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_x0_host = nullptr; return; }
+        if (cudaHostAlloc(&g_x0_host, 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) { g_x0_host = nullptr; return; }
         memset(g_x0_host, 0, 64);
         if (cudaHostGetDevicePointer(&g_x0_dev, g_x0_host, 0) != cudaSuccess) g_x0_dev = nullptr;
     });
@@ -68,7 +68,7 @@ unsigned int* x0_hint_ptr() {
 
 unsigned int* watchdog_ptr() {
     std::call_once(g_wd_once, [] {
-        if (cudaHostAlloc(&g_wd_host, 64, cudaHostAllocMapped) != cudaSuccess) { g_wd_host = nullptr; return; }
+        if (cudaHostAlloc(&g_wd_host, 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) { g_wd_host = nullptr; return; }
         memset(g_wd_host, 0, 64);
         if (cudaHostGetDevicePointer(&g_wd_dev, g_wd_host, 0) != cudaSuccess) g_wd_dev = nullptr;
     });
