@@ -428,7 +428,12 @@ int enqueue_decompress(const uint8_t* hdr, const uint32_t* table_dev, uint64_t f
     p.vrange = range_h;
     p.nz2 = 0x8000000080000000ull;
     const bool ms = (flags & HF_MS) != 0;
-    CK(launch_decode(dtype, mode, ms, p, grid, s));
+    // the decoder form follows the encoder-form hint of the stream's bound (pfpl_encode.cuh:
+    // both decoder forms decode every stream; the hint only predicts the chunks' shape)
+    bool x0 = false;
+    if (dtype == PFPL_F32 && mode == MODE_ABS && (bound == PFPL_ABS || bound == PFPL_NOA) && g_x0_host)
+        x0 = ((volatile unsigned int*)g_x0_host)[bound == PFPL_NOA ? 1 : 0] == 1u;
+    CK(launch_decode(dtype, mode, ms, x0, p, grid, s));
     g_launches += 1;
     sc->ticket_val += (uint64_t)grid * (uint64_t)decode_tickets_per_cta();   // decoder: no tickets
     return PFPL_OK;

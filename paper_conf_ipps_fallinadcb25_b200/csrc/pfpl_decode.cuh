@@ -299,7 +299,11 @@ struct VerNone {
     static __device__ __forceinline__ void flush_cta(const unsigned long long*, const DecParams&) {}
 };
 
-template <typename T, int MODE, bool MSR, bool VER = false>
+// X0: the decoder form for streams whose chunks start with a large first residual (the
+// encoder's X0 form writes them, and so does any encoder on such fields): a warp's top planes
+// in which only its first byte is non-zero are folded into thread 0 of the warp after the
+// inverse transpose instead of widening its tier.  Both forms decode every stream.
+template <typename T, int MODE, bool MSR, bool VER = false, bool X0 = false>
 __global__ void __launch_bounds__(Tr<T>::NT + 32, sizeof(T) == 4 ? PFPL_DEC_MINB : PFPL_DEC_MINB64(MODE))
 decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
     typedef typename Tr<T>::W W;
@@ -627,18 +631,45 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
 
         // ---- level 1: active planes of this warp, counts, offsets, gather ----
         int P;
+        uint64_t all;
         {
             const uint32_t a0 = S.act[lane * NWC + warp];                 // plane p = lane
             const uint32_t a1 = B == 64 ? S.act[(lane + 32) * NWC + warp] : 0u;
             const uint32_t ml = __ballot_sync(PFPL_FULL, a0 != 0);        // bit p: plane p
             const uint32_t mh = __ballot_sync(PFPL_FULL, a1 != 0);        // bit p: plane 32+p
             // bit b of `all` = bit b of the residuals active (plane B-1-b)
-            const uint64_t all = B == 32 ? (uint64_t)__brev(ml)
+            all = B == 32 ? (uint64_t)__brev(ml)
                                          : (((uint64_t)__brev(ml) << 32) | __brev(mh));
             P = all ? 64 - __clzll((long long)all) : 0;
         }
+        // X0 (f32 ABS): planes above the rest of this warp's planes in which only byte 0 of
+        // the warp's segment is non-zero (M1 segment = 01 00 .. 00): their byte carries bits of
+        // the warp's first 8 elements only, so they are counted here and OR-ed into thread 0's
+        // values after the inverse transpose, and the tier covers the other planes
+        constexpr bool kX0 = X0 && sizeof(T) == 4 && MODE == MODE_ABS;
+        uint32_t xh = 0;
+        if constexpr (kX0) {
+            const uint4 sg = *(const uint4*)(S.m1 + (B - 1 - lane) * (CW / 64) + 16 * warp);   // bit `lane`
+            const uint32_t cb = __ballot_sync(PFPL_FULL, sg.x == 1u && (sg.y | sg.z | sg.w) == 0u);
+            const uint32_t allw = (uint32_t)all;            // bit b: plane of residual bit b active
+            const uint32_t rest = allw & ~cb;
+            const int P0 = rest ? 32 - __clz(rest) : 0;
+            // the tier's planes (PFPL_DEC_TIER's widths) stay in the gather; only candidates
+            // above it are folded (each plane is counted and read exactly once)
+            const int K = P0 == 0 ? 0 : P0 <= 4 ? 4 : P0 <= 8 ? 8 : P0 <= 16 ? 16 : 32;
+            xh = allw & ~(K >= 32 ? 0xFFFFFFFFu : (1u << K) - 1u);     // all candidates (rest < 2^P0)
+            P = P0;
+        }
         uint32_t nb[64], ex[16];
         PFPL_DEC_TIER(dec1_count, S.m1, S, tid, lane, warp, nb, ex);
+        if (kX0 && xh && lane == 31) {
+            // one byte per folded plane in this warp's counts (after the row's own stores)
+#pragma unroll
+            for (int b0 = 0; b0 < 32; b0 += 4) {
+                const uint32_t nb4 = (xh >> b0) & 0xFu;
+                if (nb4) *(uint32_t*)&S.wcnt[warp][b0] += (nb4 * 0x00204081u) & 0x01010101u;
+            }
+        }
         named_sync(1, NTC);    // counts visible
         uint32_t offl, offh, n1;
         {
@@ -669,6 +700,18 @@ decode_kernel(const DecParams p, const __grid_constant__ CUtensorMap tmap) {
         if (!consistent) P = 0;           // no Z1 reads: the gather offsets are not trusted
         uint32_t lo[32], hi[32];
         PFPL_DEC_TIER(dec1_gather, lo, hi, z1, lane, nb, ex, offl, offh, S.sel);
+        if (kX0 && xh && consistent) {
+#pragma unroll 1
+            for (uint32_t mm = xh; mm; mm &= mm - 1u) {
+                const int b = __ffs(mm) - 1;
+                const uint32_t o = __shfl_sync(PFPL_FULL, offl, b);   // this warp's segment start
+                if (lane == 0) {
+                    const uint32_t v = z1[o];
+#pragma unroll
+                    for (int e = 0; e < 8; ++e) lo[e] |= ((v >> e) & 1u) << b;
+                }
+            }
+        }
 
         // ---- residual decode + delta decoder's inclusive scan ----
         W dq[32];

@@ -33,7 +33,14 @@ void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms, bool x0) {
 #else
 // decoder: (residual code, verify mode); verify is instantiated for the default residuals
 // and for zigzag residuals alike
-void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms, bool ver) {
+void* PFPL_NAME(PFPL_PREFIX, PFPL_DT, PFPL_MODE)(bool ms, bool ver, bool x0) {
+#if PFPL_DT == 0 && PFPL_MODE == 0
+    // f32 ABS (and NOA streams): the form that folds a warp's first-byte-only top planes
+    if (x0 && !ver) return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, false, true>
+                              : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, false, true>;
+#else
+    (void)x0;
+#endif
     if (ver) return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, true>
                        : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, true>;
     return ms ? (void*)PFPL_KERNEL<InstT, PFPL_MODE, true, false> : (void*)PFPL_KERNEL<InstT, PFPL_MODE, false, false>;

@@ -85,7 +85,7 @@ struct DecParams {
 // kernel launchers (pfpl_kernels.cu)
 cudaError_t launch_encode(int dtype, int mode, bool ms, bool x0, const EncParams& p, int grid,
                           cudaStream_t s);
-cudaError_t launch_decode(int dtype, int mode, bool ms, const DecParams& p, int grid,
+cudaError_t launch_decode(int dtype, int mode, bool ms, bool x0, const DecParams& p, int grid,
                           cudaStream_t s);   // p.orig != null selects the verify kernel
 int scan_grid(uint64_t C);
 cudaError_t launch_size_scan(const uint32_t* table, uint64_t C, uint64_t n, uint32_t cw,

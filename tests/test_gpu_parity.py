@@ -446,4 +446,11 @@ def test_f32_abs_both_encoder_forms(pk, orc, ms, bound):
         forms.append(pk.f32_encoder_form(bound))
         _check(pk, orc, x, bound, e, ms=ms)
     assert forms[1] == 1 and forms[3] == 0 and forms[5] == 1, forms
+    # the decoder follows the same hint (pfpl_decompress): with it at 1, decode the oracle's
+    # stream of the small-magnitude field (no foldable planes) and of the large one
+    assert pk.f32_encoder_form(bound) == 1
+    for x, e in ((xs, es), (xb, eb)):
+        s_cpu = orc.compress(x, bound, e, ms=ms)
+        y = pk.decompress(torch.frombuffer(bytearray(s_cpu), dtype=torch.uint8).cuda()).cpu().numpy()
+        assert np.array_equal(_bits(y), _bits(orc.decompress(s_cpu)))
 
