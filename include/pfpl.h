@@ -234,8 +234,9 @@ uint64_t pfpl_launch_count(void);
  * residual (taken against q[-1] = 0) in single-byte extra planes instead of widening
  * warp 0's bit-plane tier, 0 = the plain encoder.  Every f32 ABS / NOA launch leaves this
  * hint for the next one of its bound from 8 samples of its input (large first bins on a
- * smooth field -> 1).  Host-only read of mapped memory; no sync.  Returns 0 for any other
- * bound. */
+ * smooth field -> 1).  pfpl_decompress* picks its f32 decoder form from the same word of
+ * the stream's bound (both decoder forms decode every stream).  Host-only read of mapped
+ * memory; no sync.  Returns 0 for any other bound. */
 int pfpl_f32_encoder_form(int bound);
 /* Build identification string ("pfpl-b200 sm_100a ..."). */
 const char* pfpl_version(void);
